@@ -1,0 +1,97 @@
+"""ORACLE (test infrastructure only): error measures and plan invariants.
+
+* ``normwise_error``  — reading C-18 of BASELINE.json's "max relative error":
+  ``max|C_gpu - C_ref| / max(max|C_ref|, 2^-126)`` per GEMM.
+* ``coverage``        — every C element lies in exactly one tile of the plan (north_star:
+  "the invariant that every C element is covered by exactly one tile").
+* ``check_plan_invariants`` — CSR well-formedness, every tile in exactly one block, the
+  per-policy block rules of §5 (P259–270) under readings C-9 / C-10.
+"""
+from __future__ import annotations
+
+from math import ceil
+
+import numpy as np
+
+from .plan_ref import Plan, POLICY_BINARY, POLICY_THRESHOLD
+
+TOL = {"f32": 1e-5, "bf16": 2e-2, "f16": 2e-2}
+
+
+def normwise_error(c_test: np.ndarray, c_ref: np.ndarray) -> float:
+    c_test = np.asarray(c_test, np.float64)
+    c_ref = np.asarray(c_ref, np.float64)
+    if c_ref.size == 0:
+        return 0.0
+    if not np.all(np.isfinite(c_test)):
+        return float("inf")
+    den = max(float(np.max(np.abs(c_ref))), 2.0 ** -126)
+    return float(np.max(np.abs(c_test - c_ref))) / den
+
+
+def significant_rel_error(c_test, c_ref, frac: float = 1e-3) -> float:
+    """Elementwise relative error over entries with |C_ref| >= frac * max|C_ref| (C-18)."""
+    c_test = np.asarray(c_test, np.float64); c_ref = np.asarray(c_ref, np.float64)
+    if c_ref.size == 0:
+        return 0.0
+    thr = frac * float(np.max(np.abs(c_ref)))
+    m = np.abs(c_ref) >= max(thr, 2.0 ** -126)
+    if not m.any():
+        return 0.0
+    return float(np.max(np.abs(c_test[m] - c_ref[m]) / np.abs(c_ref[m])))
+
+
+def coverage(p: Plan, Ms, Ns):
+    """Per-GEMM integer maps counting how many encoded tile slots cover each C element."""
+    maps = [np.zeros((int(m), int(n)), np.int32) for m, n in zip(Ms, Ns)]
+    enc = p.enc
+    for slot in range(len(enc.GEMM)):
+        g = enc.GEMM[slot]
+        row = enc.Tiling[g] % len(p.table.rows)
+        s = p.table.rows[row]
+        y0, x0 = enc.Y[slot] * s.BY, enc.X[slot] * s.BX
+        maps[g][y0:y0 + s.BY, x0:x0 + s.BX] += 1
+    return maps
+
+
+def check_plan_invariants(p: Plan, Ms, Ns, Ks, policy: int, theta: int) -> None:
+    enc = p.enc
+    n_tiles = len(p.tiles)
+    assert enc.Tile[0] == 0 and enc.Tile[-1] == n_tiles == len(enc.GEMM)
+    assert all(a <= b for a, b in zip(enc.Tile, enc.Tile[1:])), "Tile[] must be monotone"
+    assert all(b > a for a, b in zip(enc.Tile, enc.Tile[1:])), "no empty block"
+    seen = sorted(t for blk in p.blocks for t in blk)
+    assert seen == list(range(n_tiles)), "every tile in exactly one block"
+    for g, (m, n) in enumerate(zip(Ms, Ns)):
+        row = enc.Tiling[g] % len(p.table.rows)
+        s = p.table.rows[row]
+        if m > 0 and n > 0:
+            cnt = sum(1 for t in p.tiles if t.gemm == g)
+            assert cnt == ceil(m / s.BY) * ceil(n / s.BX)
+    for cov in coverage(p, Ms, Ns):
+        assert cov.size == 0 or (cov.min() == 1 and cov.max() == 1), "each C element in exactly one tile"
+    Kt = [t.K for t in p.tiles]
+    if policy == POLICY_BINARY:
+        for blk in p.blocks:
+            assert 1 <= len(blk) <= 2
+            if len(blk) == 2:
+                assert Kt[blk[0]] <= Kt[blk[1]] < theta
+    if policy == POLICY_THRESHOLD:
+        # a block with more than one tile was opened in fill mode: its K-sum reached θ
+        # only with its last tile (or tiles ran out at the end of the list)
+        last = len(p.blocks) - 1
+        for b, blk in enumerate(p.blocks):
+            if len(blk) > 1:
+                ks = [Kt[t] for t in blk]
+                assert sum(ks[:-1]) < theta
+                assert sum(ks) >= theta or b == last or blk[-1] == n_tiles - 1
+    # tiler trace: each round's strategy per GEMM is at least as late in priority order
+    # (tile area never shrinks); the final strategy fits the GEMM unless nothing fits (C-1, C-4)
+    tr = p.tiling.trace
+    pos = {r: i for i, r in enumerate(p.table.order())}
+    for (r0, _, _), (r1, _, _) in zip(tr, tr[1:]):
+        assert all(pos[b] >= pos[a] for a, b in zip(r0, r1))
+    for g, (m, n) in enumerate(zip(Ms, Ns)):
+        s = p.table.rows[p.tiling.rows[g]]
+        fits_any = any(q.BY <= m and q.BX <= n for q in p.table.rows)
+        assert (s.BY <= m and s.BX <= n) or (not fits_any and p.tiling.rows[g] == p.table.order()[0])

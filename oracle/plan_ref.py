@@ -1,0 +1,283 @@
+"""ORACLE (test infrastructure only): reference tiling engine, batching engine, encoding, sharder.
+
+Plain Python, step by step in the paper's order and notation.  Shares no code, table or
+constant generator with the C++ planner in ``paper_conf_ppopp_li0yjl19_b200/csrc``; the
+tables below are restated here from PAPER.md Table 2 (P204–214) and DESIGN.md §4.
+
+Readings of silent / garbled passages are numbered C-1 … C-24 as in DESIGN.md §3.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+from math import ceil
+from typing import List, Sequence, Tuple
+
+
+# ----------------------------------------------------------------------------------------
+# Strategy tables
+# ----------------------------------------------------------------------------------------
+@dataclass(frozen=True)
+class Strategy:
+    name: str
+    BY: int      # tile rows    (along M)
+    BX: int      # tile columns (along N)
+    BK: int      # K step of one main-loop iteration
+
+
+@dataclass(frozen=True)
+class Table:
+    name: str
+    rows: Tuple[Strategy, ...]           # table row order (ids are derived from it)
+    versions: Tuple[int, ...]            # thread counts T, first = preferred (more TLP)
+    tlp_threshold: int                   # default TLP threshold (P253, P290)
+    theta: int                           # default batching threshold θ (P259, P290)
+
+    def order(self) -> List[int]:
+        """Priority order: smaller tile first (P249); ties by table row (reading C-3)."""
+        return sorted(range(len(self.rows)), key=lambda r: (self.rows[r].BY * self.rows[r].BX, r))
+
+    def strategy_id(self, row: int, T: int) -> int:
+        """Reading C-14: id = version_index * n_rows + row ("0-11" for Table 2, P282)."""
+        return self.versions.index(T) * len(self.rows) + row
+
+
+# PAPER.md Table 2 (P204–214), the V100 profile: six shapes, BK = 8 (P243),
+# 256- and 128-thread versions (P181, P198); TLP threshold 65536 and θ = 256 (P255, P290).
+V100 = Table("v100_table2", (
+    Strategy("small", 16, 16, 8), Strategy("medium", 32, 32, 8), Strategy("large", 64, 64, 8),
+    Strategy("tall", 128, 64, 8), Strategy("wide", 64, 128, 8), Strategy("huge", 128, 128, 8)),
+    versions=(256, 128), tlp_threshold=65536, theta=256)
+
+# B200 FFMA (fp32) profile: the Table 2 shapes and sub-tiles are an FFMA design and are
+# kept; the platform constants are re-set for 148 SMs (reading C-22).
+B200_F32 = Table("b200_ffma", V100.rows, versions=(256, 128), tlp_threshold=131072, theta=256)
+
+# B200 tcgen05 (bf16/fp16) profile: C-tile shapes sized for tcgen05.mma
+# (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16).  One kernel "version" with
+# T = 256 threads (8 warps), so the paper's version switch is a no-op for this table.
+B200_TC = Table("b200_tcgen05", (
+    Strategy("s", 64, 32, 64), Strategy("m", 64, 64, 64), Strategy("t", 128, 64, 64),
+    Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("h", 128, 256, 64)),
+    versions=(256,), tlp_threshold=4 * 148 * 256, theta=512)
+
+TABLES = {1: V100, 2: B200_F32, 3: B200_TC}
+
+
+# ----------------------------------------------------------------------------------------
+# Tiling engine (§4.2.3, P245–255)
+# ----------------------------------------------------------------------------------------
+def tlp(Ms, Ns, rows: Sequence[int], table: Table, T: int) -> int:
+    """Eq. 1 (P220): TLP = sum_i (M_i*N_i)/(BY_i*BX_i) * T, tiles counted with ceil (C-5)."""
+    total = 0
+    for M, N, r in zip(Ms, Ns, rows):
+        s = table.rows[r]
+        total += ceil(M / s.BY) * ceil(N / s.BX)
+    return total * T
+
+
+@dataclass
+class TilingResult:
+    rows: List[int]            # chosen table row per GEMM
+    T: int                     # chosen version (threads per block)
+    trace: List[Tuple[List[int], int, int]] = field(default_factory=list)  # (rows, T, TLP) per round
+
+    def ids(self, table: Table) -> List[int]:
+        return [table.strategy_id(r, self.T) for r in self.rows]
+
+
+def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None) -> TilingResult:
+    """The three steps and two exceptions of P249–253.
+
+    1. Per GEMM, a priority queue of the strategies with BY <= M and BX <= N (C-1),
+       smallest first (P249); if none fits, the smallest strategy alone (C-4).
+    2. Take one strategy per GEMM: pop, or top if only one is left (exception 1, C-2);
+       TLP by Eq. 1 with the current version T.
+    3. If TLP > threshold (strict, C-6) repeat step 2; otherwise this is the solution.
+       Exception 2 (C-7): if step 2 is to be repeated while every queue holds a single
+       strategy, switch to the second version (128 threads) and repeat step 2 once more;
+       if no further version exists, stop with the current solution.
+    """
+    thr = table.tlp_threshold if threshold is None else threshold
+    order = table.order()
+    queues = []
+    for M, N in zip(Ms, Ns):
+        q = [r for r in order if table.rows[r].BY <= M and table.rows[r].BX <= N]
+        queues.append(q if q else [order[0]])
+    vi = 0
+    T = table.versions[vi]
+    trace = []
+    while True:
+        cur = [q.pop(0) if len(q) > 1 else q[0] for q in queues]       # step 2
+        t = tlp(Ms, Ns, cur, table, T)
+        trace.append((list(cur), T, t))
+        if t <= thr:                                                   # step 3
+            return TilingResult(cur, T, trace)
+        if all(len(q) == 1 for q in queues):                           # exception 2
+            if vi + 1 >= len(table.versions):
+                return TilingResult(cur, T, trace)
+            vi += 1
+            T = table.versions[vi]
+
+
+# ----------------------------------------------------------------------------------------
+# Tile enumeration (P133–135, P157, P284)
+# ----------------------------------------------------------------------------------------
+@dataclass(frozen=True)
+class Tile:
+    gemm: int
+    y: int        # tile row index along M   (C-13)
+    x: int        # tile column index along N
+    K: int        # K-workload of the tile = K of its GEMM (C-11)
+
+
+def enumerate_tiles(Ms, Ns, Ks, rows: Sequence[int], table: Table) -> List[Tile]:
+    """GEMM-major, then row-major (y, x): ceil(M/BY) x ceil(N/BX) tiles per GEMM."""
+    tiles = []
+    for g, (M, N, K, r) in enumerate(zip(Ms, Ns, Ks, rows)):
+        s = table.rows[r]
+        if M <= 0 or N <= 0:
+            continue
+        for y in range(ceil(M / s.BY)):
+            for x in range(ceil(N / s.BX)):
+                tiles.append(Tile(g, y, x, int(K)))
+    return tiles
+
+
+# ----------------------------------------------------------------------------------------
+# Batching engine (§5, P259–270)
+# ----------------------------------------------------------------------------------------
+def threshold_batching(tiles: Sequence[Tile], T: int, tlp_threshold: int, theta: int) -> List[List[int]]:
+    """Threshold batching, TLP first (P261; garbled passage, reading C-9).
+
+    Before opening each new block: TLP = (#unassigned tiles + #assigned blocks) * T.
+    If TLP > threshold / 2, fill the new block with tiles (enumeration order) until the sum
+    of their K is not less than θ; otherwise every remaining tile gets its own block.
+    """
+    n = len(tiles)
+    blocks: List[List[int]] = []
+    i = 0
+    while i < n:
+        t = ((n - i) + len(blocks)) * T
+        if t > tlp_threshold / 2:
+            blk, sk = [], 0
+            while i < n and sk < theta:
+                blk.append(i)
+                sk += tiles[i].K
+                i += 1
+            blocks.append(blk)
+        else:
+            while i < n:
+                blocks.append([i])
+                i += 1
+    return blocks
+
+
+def binary_batching(tiles: Sequence[Tile], theta: int) -> List[List[int]]:
+    """Binary batching, ILP first (P263–270, Eq. 5; reading C-10).
+
+    Sort tiles by K ascending (stable: ties keep enumeration order); repeatedly pair the
+    first (minimal K) with the last (maximal K).  A last tile with K >= θ goes alone (a
+    pair containing it can only increase Eq. 5's objective); an odd middle tile goes alone.
+    """
+    order = sorted(range(len(tiles)), key=lambda t: (tiles[t].K, t))
+    blocks: List[List[int]] = []
+    lo, hi = 0, len(order) - 1
+    while lo <= hi:
+        if lo == hi:
+            blocks.append([order[lo]])
+            break
+        if tiles[order[hi]].K >= theta:
+            blocks.append([order[hi]])
+            hi -= 1
+        else:
+            blocks.append([order[lo], order[hi]])
+            lo += 1
+            hi -= 1
+    return blocks
+
+
+def no_batching(tiles: Sequence[Tile]) -> List[List[int]]:
+    """One tile per block (the un-batched baseline: "a thread block is responsible for a single tile", P259)."""
+    return [[i] for i in range(len(tiles))]
+
+
+def eq5_objective(tiles: Sequence[Tile], blocks: Sequence[Sequence[int]], theta: int) -> int:
+    """Eq. 5 (P267): sum over two-tile blocks of |K_i + K_j - θ|."""
+    return sum(abs(tiles[b[0]].K + tiles[b[1]].K - theta) for b in blocks if len(b) == 2)
+
+
+# ----------------------------------------------------------------------------------------
+# Programming interface: the five auxiliary arrays (§6, P282–284, Fig. 6 / Fig. 7)
+# ----------------------------------------------------------------------------------------
+@dataclass
+class Encoded:
+    Tile: List[int]          # CSR offsets, Block_NUM + 1 entries
+    GEMM: List[int]          # per tile slot: source GEMM
+    Y: List[int]             # per tile slot: tile row index
+    X: List[int]             # per tile slot: tile column index
+    Tiling: List[int]        # per GEMM: strategy id (C-12)
+
+
+def encode(tiles: Sequence[Tile], blocks: Sequence[Sequence[int]], gemm_strategy_ids: Sequence[int]) -> Encoded:
+    """Block b owns tile slots [Tile[b], Tile[b+1]) (P282); slots follow block order."""
+    Tl, G, Y, X = [0], [], [], []
+    for blk in blocks:
+        for t in blk:
+            G.append(tiles[t].gemm)
+            Y.append(tiles[t].y)
+            X.append(tiles[t].x)
+        Tl.append(len(G))
+    return Encoded(Tl, G, Y, X, list(gemm_strategy_ids))
+
+
+# ----------------------------------------------------------------------------------------
+# Whole plan
+# ----------------------------------------------------------------------------------------
+POLICY_THRESHOLD, POLICY_BINARY, POLICY_NONE = 0, 1, 2
+
+
+@dataclass
+class Plan:
+    table: Table
+    tiling: TilingResult
+    tiles: List[Tile]
+    blocks: List[List[int]]
+    enc: Encoded
+
+
+def plan(Ms, Ns, Ks, table: Table, policy: int = POLICY_THRESHOLD,
+         tlp_threshold: int | None = None, theta: int | None = None) -> Plan:
+    thr = table.tlp_threshold if tlp_threshold is None else tlp_threshold
+    th = table.theta if theta is None else theta
+    Ms = [int(v) for v in Ms]; Ns = [int(v) for v in Ns]; Ks = [int(v) for v in Ks]
+    tr = tiling_engine(Ms, Ns, table, thr)
+    tiles = enumerate_tiles(Ms, Ns, Ks, tr.rows, table)
+    if policy == POLICY_THRESHOLD:
+        blocks = threshold_batching(tiles, tr.T, thr, th)
+    elif policy == POLICY_BINARY:
+        blocks = binary_batching(tiles, th)
+    elif policy == POLICY_NONE:
+        blocks = no_batching(tiles)
+    else:
+        raise ValueError(policy)
+    enc = encode(tiles, blocks, tr.ids(table))
+    return Plan(table, tr, tiles, blocks, enc)
+
+
+# ----------------------------------------------------------------------------------------
+# Multi-GPU: FLOP-balanced GEMM -> rank assignment (BASELINE.json north_star; C-23)
+# ----------------------------------------------------------------------------------------
+def shard_lpt(Ms, Ns, Ks, n_ranks: int) -> List[int]:
+    """Longest-processing-time first on work 2*M*N*K: GEMMs by (-work, index) each go to
+    the least-loaded rank, ties to the lowest rank."""
+    if n_ranks <= 0:
+        raise ValueError("n_ranks must be positive")
+    work = [2 * int(m) * int(n) * int(k) for m, n, k in zip(Ms, Ns, Ks)]
+    order = sorted(range(len(work)), key=lambda g: (-work[g], g))
+    load = [0] * n_ranks
+    rank_of = [0] * len(work)
+    for g in order:
+        r = min(range(n_ranks), key=lambda q: (load[q], q))
+        rank_of[g] = r
+        load[r] += work[g]
+    return rank_of
