@@ -1,0 +1,520 @@
+// C-ABI of include/vbgemm.h: plan lifetime, validation, device descriptor upload,
+// tensor-map encoding, exec dispatch, export of the device plan, input fill.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/vbgemm.h"
+#include "plan_types.h"
+#include "planner.h"
+#include "tables.h"
+
+namespace vb {
+cudaError_t launch_f32(const F32Args &args, int n_blocks, int version_T, cudaStream_t stream);
+cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, uint8_t *tmaps, const void *const *A,
+                      const void *const *B, void *const *C, const GemmParam *gemms, int batch, cudaStream_t stream);
+cudaError_t tc_configure();
+size_t tc_smem_bytes();
+cudaError_t launch_fill(int dt, int batch, const int32_t *rows, const int32_t *cols, const int32_t *ld,
+                        void *const *ptrs, const int64_t *gemm_id, uint64_t seed, int operand, int64_t total_elems,
+                        cudaStream_t stream);
+cudaError_t launch_alpha_beta(int batch, const int64_t *gemm_id, uint64_t seed, float *alpha, float *beta,
+                              cudaStream_t stream);
+}  // namespace vb
+
+using namespace vb;
+
+static thread_local std::string g_last_error;
+
+static vb_status fail(vb_status s, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return s;
+}
+static vb_status cuda_fail(cudaError_t e, const char *what) {
+  return fail(VB_ERR_CUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+struct vb_plan {
+  int device = -1;
+  vb_dtype dt = VB_F32;
+  int batch = 0;
+  const TableDef *table = nullptr;
+  int policy = 0;
+  TilingOut tiling;
+  std::vector<int32_t> block_ptr;     // Tile[]
+  std::vector<TileSlot> slots;        // GEMM[], Y[], X[]
+  std::vector<GemmParam> gemms;       // sizes + Tiling[] (row)
+  // device side
+  void *d_ws = nullptr;
+  size_t ws_bytes = 0;
+  int32_t *d_block_ptr = nullptr;
+  TileSlot *d_slots = nullptr;
+  GemmParam *d_gemms = nullptr;
+  uint8_t *d_tmaps = nullptr;
+  int32_t *d_counter = nullptr;
+  int sm_count = 0;
+  ~vb_plan() {
+    if (d_ws) {
+      int prev = 0;
+      cudaGetDevice(&prev);
+      cudaSetDevice(device);
+      cudaFree(d_ws);
+      cudaSetDevice(prev);
+    }
+  }
+};
+
+static int elem_bytes(vb_dtype dt) { return dt == VB_F32 ? 4 : 2; }
+
+static int64_t cdiv64(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// ------------------------------------------------------------------------ tensor maps
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+static CUtensorMapSwizzle swizzle_of(int bytes) {
+  return bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : (bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B);
+}
+
+static vb_status encode_2d(CUtensorMap *m, vb_dtype dt, void *addr, uint64_t inner, uint64_t outer, uint64_t ld_elems,
+                           uint32_t box_inner, uint32_t box_outer, int swz_bytes) {
+  auto enc = get_encode();
+  if (!enc) return fail(VB_ERR_CUDA, "cuTensorMapEncodeTiled entry point unavailable");
+  const CUtensorMapDataType t = dt == VB_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {ld_elems * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(m, t, 2, addr, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_of(swz_bytes),
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS)
+    return fail(VB_ERR_INTERNAL, "cuTensorMapEncodeTiled failed (%d) dims %llu x %llu ld %llu box %u x %u", (int)r,
+                (unsigned long long)inner, (unsigned long long)outer, (unsigned long long)ld_elems, box_inner,
+                box_outer);
+  return VB_OK;
+}
+
+// ------------------------------------------------------------------------ validation
+static vb_status validate_shapes(vb_dtype dt, int32_t batch, const int32_t *M, const int32_t *N, const int32_t *K,
+                                 const int32_t *lda, const int32_t *ldb, const int32_t *ldc) {
+  if (batch < 0) return fail(VB_ERR_INVALID_ARG, "batch < 0");
+  if (dt != VB_F32 && dt != VB_BF16 && dt != VB_F16) return fail(VB_ERR_INVALID_ARG, "unknown dtype %d", (int)dt);
+  if (batch > 0 && (!M || !N || !K || !lda || !ldb || !ldc)) return fail(VB_ERR_INVALID_ARG, "null size array");
+  const int es = elem_bytes(dt);
+  for (int i = 0; i < batch; ++i) {
+    if (M[i] < 0 || N[i] < 0 || K[i] < 0) return fail(VB_ERR_INVALID_ARG, "GEMM %d: negative size", i);
+    if (M[i] > (1 << 20) || N[i] > (1 << 20)) return fail(VB_ERR_INVALID_ARG, "GEMM %d: M or N above 2^20", i);
+    if (M[i] == 0 || N[i] == 0) continue;
+    if (ldc[i] < N[i] || (K[i] > 0 && (lda[i] < K[i] || ldb[i] < N[i])))
+      return fail(VB_ERR_INVALID_ARG, "GEMM %d: leading dimension below the row length", i);
+    if (((int64_t)ldc[i] * es) % 16 || (K[i] > 0 && (((int64_t)lda[i] * es) % 16 || ((int64_t)ldb[i] * es) % 16)))
+      return fail(VB_ERR_ALIGNMENT, "GEMM %d: ld * sizeof(elem) must be a multiple of 16 bytes", i);
+  }
+  return VB_OK;
+}
+
+static const TableDef *resolve_table(vb_dtype dt, int table_id) {
+  if (table_id == VB_TABLE_DEFAULT) table_id = dt == VB_F32 ? VB_TABLE_B200_FFMA : VB_TABLE_B200_TC;
+  return table_by_id(table_id);
+}
+
+static bool table_runs_on(const TableDef *t, vb_dtype dt) {
+  if (dt == VB_F32) return t->id == VB_TABLE_V100 || t->id == VB_TABLE_B200_FFMA;
+  return t->id == VB_TABLE_B200_TC;
+}
+
+// ------------------------------------------------------------------------ device upload
+static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const int32_t *K, const int32_t *lda,
+                        const int32_t *ldb, const int32_t *ldc) {
+  cudaError_t e = cudaSetDevice(p->device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+  cudaDeviceProp prop;
+  e = cudaGetDeviceProperties(&prop, p->device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceProperties");
+  if (prop.major != 10 || prop.minor != 0)
+    return fail(VB_ERR_UNSUPPORTED, "device %d is sm_%d%d; this library is built for sm_100a", p->device, prop.major,
+                prop.minor);
+  p->sm_count = prop.multiProcessorCount;
+  const bool tc = p->dt != VB_F32;
+  auto align_up = [](size_t v, size_t a) { return (v + a - 1) / a * a; };
+  size_t off = 0;
+  const size_t o_bp = off;
+  off = align_up(off + p->block_ptr.size() * sizeof(int32_t), 256);
+  const size_t o_sl = off;
+  off = align_up(off + std::max<size_t>(p->slots.size(), 1) * sizeof(TileSlot), 256);
+  const size_t o_gp = off;
+  off = align_up(off + std::max<size_t>(p->gemms.size(), 1) * sizeof(GemmParam), 256);
+  const size_t o_ct = off;
+  off = align_up(off + 256, 256);
+  const size_t o_tm = off;
+  if (tc) off = align_up(off + (size_t)p->batch * 3 * 128, 256);
+  p->ws_bytes = off;
+  e = cudaMalloc(&p->d_ws, p->ws_bytes);
+  if (e != cudaSuccess) {
+    p->d_ws = nullptr;
+    return fail(VB_ERR_OOM, "cudaMalloc(%zu) for plan workspace: %s", p->ws_bytes, cudaGetErrorString(e));
+  }
+  uint8_t *base = static_cast<uint8_t *>(p->d_ws);
+  p->d_block_ptr = reinterpret_cast<int32_t *>(base + o_bp);
+  p->d_slots = reinterpret_cast<TileSlot *>(base + o_sl);
+  p->d_gemms = reinterpret_cast<GemmParam *>(base + o_gp);
+  p->d_counter = reinterpret_cast<int32_t *>(base + o_ct);
+  p->d_tmaps = tc ? base + o_tm : nullptr;
+
+  std::vector<uint8_t> host(p->ws_bytes, 0);
+  memcpy(host.data() + o_bp, p->block_ptr.data(), p->block_ptr.size() * sizeof(int32_t));
+  if (!p->slots.empty()) memcpy(host.data() + o_sl, p->slots.data(), p->slots.size() * sizeof(TileSlot));
+  if (!p->gemms.empty()) memcpy(host.data() + o_gp, p->gemms.data(), p->gemms.size() * sizeof(GemmParam));
+  if (tc) {
+    e = tc_configure();
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(tc kernel smem)");
+    // Per-GEMM tensor maps encoded now with a placeholder address; exec patches the address.
+    CUtensorMap *maps = reinterpret_cast<CUtensorMap *>(host.data() + o_tm);
+    for (int i = 0; i < p->batch; ++i) {
+      if (M[i] == 0 || N[i] == 0) continue;
+      const StrategyRow &s = p->table->rows[p->tiling.row[i]];
+      const TcGeom g = tc_geom(s.BY, s.BX);
+      vb_status st;
+      if (K[i] > 0) {
+        st = encode_2d(&maps[3 * i + 0], p->dt, p->d_ws, (uint64_t)K[i], (uint64_t)M[i], (uint64_t)lda[i], 64,
+                       (uint32_t)s.BY, 128);
+        if (st != VB_OK) return st;
+        st = encode_2d(&maps[3 * i + 1], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)K[i], (uint64_t)ldb[i],
+                       (uint32_t)(g.b_swz / 2), 64, g.b_swz);
+        if (st != VB_OK) return st;
+      }
+      st = encode_2d(&maps[3 * i + 2], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)M[i], (uint64_t)ldc[i],
+                     (uint32_t)g.c_cols, (uint32_t)s.BY, g.c_swz);
+      if (st != VB_OK) return st;
+    }
+  }
+  e = cudaMemcpy(p->d_ws, host.data(), p->ws_bytes, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy(plan descriptors)");
+  return VB_OK;
+}
+
+// ------------------------------------------------------------------------ plan building
+static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, const int32_t *K, const int32_t *lda,
+                             const int32_t *ldb, const int32_t *ldc, const std::vector<TileRec> &tiles,
+                             const Schedule &sch) {
+  p->block_ptr = sch.block_ptr;
+  p->slots.resize(sch.slot_tile.size());
+  for (size_t s = 0; s < sch.slot_tile.size(); ++s) {
+    const TileRec &t = tiles[(size_t)sch.slot_tile[s]];
+    if (t.y > 0xFFFF || t.x > 0xFFFF) return fail(VB_ERR_INVALID_ARG, "tile index above 65535");
+    p->slots[s] = TileSlot{(uint32_t)t.gemm, (uint16_t)t.y, (uint16_t)t.x};
+  }
+  p->gemms.resize((size_t)p->batch);
+  for (int i = 0; i < p->batch; ++i) {
+    const StrategyRow &s = p->table->rows[p->tiling.row[i]];
+    GemmParam &g = p->gemms[(size_t)i];
+    g.M = M[i];
+    g.N = N[i];
+    g.K = K[i];
+    g.lda = lda[i];
+    g.ldb = ldb[i];
+    g.ldc = ldc[i];
+    g.row = p->tiling.row[i] | (s.BY << 8) | (s.BX << 16);
+    g.kblocks = (int32_t)cdiv64(K[i], s.BK);
+  }
+  if (p->device >= 0) return upload(p, M, N, K, lda, ldb, ldc);
+  return VB_OK;
+}
+
+extern "C" vb_status vb_plan_vbatched(int device, vb_dtype dt, int32_t batch, const int32_t *M, const int32_t *N,
+                                      const int32_t *K, const int32_t *lda, const int32_t *ldb, const int32_t *ldc,
+                                      vb_policy policy, const vb_tuning *tuning, vb_plan_t *out) {
+  try {
+    if (!out) return fail(VB_ERR_INVALID_ARG, "out is null");
+    *out = nullptr;
+    vb_status st = validate_shapes(dt, batch, M, N, K, lda, ldb, ldc);
+    if (st != VB_OK) return st;
+    if (policy != VB_BATCH_THRESHOLD && policy != VB_BATCH_BINARY && policy != VB_BATCH_NONE)
+      return fail(VB_ERR_INVALID_ARG, "unknown policy %d", (int)policy);
+    const TableDef *t = resolve_table(dt, tuning ? tuning->table_id : 0);
+    if (!t) return fail(VB_ERR_INVALID_ARG, "unknown table id %d", tuning ? tuning->table_id : -1);
+    if (device >= 0 && !table_runs_on(t, dt))
+      return fail(VB_ERR_UNSUPPORTED, "table %s has no kernel for this dtype", t->name);
+    const int64_t thr = (tuning && tuning->tlp_threshold > 0) ? tuning->tlp_threshold : t->tlp_threshold;
+    const int theta = (tuning && tuning->theta > 0) ? tuning->theta : t->theta;
+    vb_plan *p = new vb_plan();
+    p->device = device;
+    p->dt = dt;
+    p->batch = batch;
+    p->table = t;
+    p->policy = (int)policy;
+    p->tiling = tiling_engine(M, N, batch, *t, thr);
+    if (batch == 0) p->tiling.version_T = t->versions[0];
+    const std::vector<TileRec> tiles = enumerate_tiles(M, N, K, batch, p->tiling.row, *t);
+    if (tiles.size() > (size_t)INT32_MAX) {
+      delete p;
+      return fail(VB_ERR_INVALID_ARG, "more than 2^31 tiles");
+    }
+    Schedule sch = policy == VB_BATCH_THRESHOLD ? batch_threshold(tiles, p->tiling.version_T, thr, theta)
+                   : policy == VB_BATCH_BINARY  ? batch_binary(tiles, theta)
+                                                : batch_none(tiles);
+    st = finish_plan(p, M, N, K, lda, ldb, ldc, tiles, sch);
+    if (st != VB_OK) {
+      delete p;
+      return st;
+    }
+    *out = p;
+    return VB_OK;
+  } catch (const std::bad_alloc &) {
+    return fail(VB_ERR_OOM, "host allocation failed");
+  } catch (...) {
+    return fail(VB_ERR_INTERNAL, "unexpected exception");
+  }
+}
+
+extern "C" vb_status vb_plan_from_schedule(int device, vb_dtype dt, int32_t batch, const int32_t *M, const int32_t *N,
+                                           const int32_t *K, const int32_t *lda, const int32_t *ldb,
+                                           const int32_t *ldc, int32_t table_id, const int32_t *gemm_row,
+                                           int32_t version_T, int32_t n_blocks, const int32_t *block_ptr,
+                                           const int32_t *tile_gemm, const int32_t *tile_y, const int32_t *tile_x,
+                                           vb_plan_t *out) {
+  try {
+    if (!out) return fail(VB_ERR_INVALID_ARG, "out is null");
+    *out = nullptr;
+    vb_status st = validate_shapes(dt, batch, M, N, K, lda, ldb, ldc);
+    if (st != VB_OK) return st;
+    const TableDef *t = resolve_table(dt, table_id);
+    if (!t) return fail(VB_ERR_INVALID_ARG, "unknown table id %d", table_id);
+    if (device >= 0 && !table_runs_on(t, dt))
+      return fail(VB_ERR_UNSUPPORTED, "table %s has no kernel for this dtype", t->name);
+    bool vok = false;
+    for (int v = 0; v < t->n_versions; ++v) vok |= (t->versions[v] == version_T);
+    if (!vok) return fail(VB_ERR_INVALID_ARG, "version_T %d not in table %s", version_T, t->name);
+    if (n_blocks < 0 || !block_ptr || (batch > 0 && !gemm_row)) return fail(VB_ERR_INVALID_ARG, "null schedule");
+    if (block_ptr[0] != 0) return fail(VB_ERR_INVALID_ARG, "block_ptr[0] must be 0");
+    for (int b = 0; b < n_blocks; ++b)
+      if (block_ptr[b + 1] < block_ptr[b]) return fail(VB_ERR_INVALID_ARG, "block_ptr not monotone at %d", b);
+    const int64_t n_slots = block_ptr[n_blocks];
+    if (n_slots > 0 && (!tile_gemm || !tile_y || !tile_x)) return fail(VB_ERR_INVALID_ARG, "null tile arrays");
+    std::vector<int64_t> tile_base((size_t)batch + 1, 0);
+    for (int i = 0; i < batch; ++i) {
+      if (gemm_row[i] < 0 || gemm_row[i] >= t->n_rows) return fail(VB_ERR_INVALID_ARG, "GEMM %d: bad row", i);
+      const StrategyRow &s = t->rows[gemm_row[i]];
+      const int64_t n = (M[i] > 0 && N[i] > 0) ? cdiv64(M[i], s.BY) * cdiv64(N[i], s.BX) : 0;
+      tile_base[(size_t)i + 1] = tile_base[(size_t)i] + n;
+    }
+    if (tile_base[(size_t)batch] != n_slots)
+      return fail(VB_ERR_INVALID_ARG, "schedule has %lld slots, the tiling has %lld tiles", (long long)n_slots,
+                  (long long)tile_base[(size_t)batch]);
+    std::vector<uint8_t> seen((size_t)n_slots, 0);
+    std::vector<TileRec> tiles((size_t)n_slots);
+    for (int64_t s = 0; s < n_slots; ++s) {
+      const int g = tile_gemm[s];
+      if (g < 0 || g >= batch) return fail(VB_ERR_INVALID_ARG, "slot %lld: bad GEMM id", (long long)s);
+      const StrategyRow &r = t->rows[gemm_row[g]];
+      const int64_t gy = cdiv64(M[g], r.BY), gx = cdiv64(N[g], r.BX);
+      if (tile_y[s] < 0 || tile_y[s] >= gy || tile_x[s] < 0 || tile_x[s] >= gx)
+        return fail(VB_ERR_INVALID_ARG, "slot %lld: tile outside GEMM %d", (long long)s, g);
+      const int64_t id = tile_base[(size_t)g] + (int64_t)tile_y[s] * gx + tile_x[s];
+      if (seen[(size_t)id]++) return fail(VB_ERR_INVALID_ARG, "slot %lld: tile covered twice", (long long)s);
+      tiles[(size_t)s] = TileRec{g, tile_y[s], tile_x[s], K[g]};
+    }
+    vb_plan *p = new vb_plan();
+    p->device = device;
+    p->dt = dt;
+    p->batch = batch;
+    p->table = t;
+    p->policy = -1;
+    p->tiling.row.assign(gemm_row, gemm_row + batch);
+    p->tiling.version_T = version_T;
+    Schedule sch;
+    sch.block_ptr.assign(block_ptr, block_ptr + n_blocks + 1);
+    sch.slot_tile.resize((size_t)n_slots);
+    for (int64_t s = 0; s < n_slots; ++s) sch.slot_tile[(size_t)s] = (int32_t)s;
+    st = finish_plan(p, M, N, K, lda, ldb, ldc, tiles, sch);
+    if (st != VB_OK) {
+      delete p;
+      return st;
+    }
+    *out = p;
+    return VB_OK;
+  } catch (const std::bad_alloc &) {
+    return fail(VB_ERR_OOM, "host allocation failed");
+  } catch (...) {
+    return fail(VB_ERR_INTERNAL, "unexpected exception");
+  }
+}
+
+extern "C" vb_status vb_exec_vbatched(vb_plan_t p, const void *const *A, const void *const *B, void *const *C,
+                                      const float *alpha, const float *beta, void *stream) {
+  if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
+  if (p->device < 0) return fail(VB_ERR_UNSUPPORTED, "host-only plan cannot be executed");
+  if (p->batch == 0) return VB_OK;
+  if (!A || !B || !C || !alpha || !beta) return fail(VB_ERR_INVALID_ARG, "null argument array");
+  int cur = -1;
+  cudaGetDevice(&cur);
+  if (cur != p->device) {
+    cudaError_t e = cudaSetDevice(p->device);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+  }
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const int n_blocks = (int)p->block_ptr.size() - 1;
+  cudaError_t e;
+  if (p->dt == VB_F32) {
+    F32Args a{p->d_block_ptr, p->d_slots, p->d_gemms, reinterpret_cast<const float *const *>(A),
+              reinterpret_cast<const float *const *>(B), reinterpret_cast<float *const *>(C), alpha, beta};
+    e = launch_f32(a, n_blocks, p->tiling.version_T, s);
+  } else {
+    TcArgs a{p->d_block_ptr, p->d_slots, p->d_gemms, p->d_tmaps, C, alpha, beta, p->d_counter, n_blocks};
+    const int grid = std::min(n_blocks, p->sm_count);
+    e = launch_tc(a, grid, p->dt == VB_BF16, p->d_tmaps, A, B, C, p->d_gemms, p->batch, s);
+  }
+  if (cur != p->device && cur >= 0) cudaSetDevice(cur);
+  if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+  return VB_OK;
+}
+
+extern "C" vb_status vb_plan_info(vb_plan_t p, int64_t *n_tiles, int64_t *n_blocks, int64_t *workspace_bytes,
+                                  int32_t *version_T, int32_t *launches_per_exec) {
+  if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
+  if (n_tiles) *n_tiles = (int64_t)p->slots.size();
+  if (n_blocks) *n_blocks = (int64_t)p->block_ptr.size() - 1;
+  if (workspace_bytes) *workspace_bytes = (int64_t)p->ws_bytes;
+  if (version_T) *version_T = p->tiling.version_T;
+  if (launches_per_exec) {
+    const bool any = p->block_ptr.size() > 1;
+    *launches_per_exec = p->batch == 0 ? 0 : (p->dt == VB_F32 ? (any ? 1 : 0) : (any ? 2 : 1));
+  }
+  return VB_OK;
+}
+
+extern "C" vb_status vb_plan_export(vb_plan_t p, int32_t *block_ptr, int32_t *tile_gemm, int32_t *tile_y,
+                                    int32_t *tile_x, int32_t *gemm_strategy) {
+  if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
+  std::vector<int32_t> bp = p->block_ptr;
+  std::vector<TileSlot> sl = p->slots;
+  std::vector<GemmParam> gm = p->gemms;
+  if (p->device >= 0) {   // decode what the kernel will actually walk
+    int cur = -1;
+    cudaGetDevice(&cur);
+    cudaSetDevice(p->device);
+    cudaError_t e = cudaMemcpy(bp.data(), p->d_block_ptr, bp.size() * sizeof(int32_t), cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess && !sl.empty())
+      e = cudaMemcpy(sl.data(), p->d_slots, sl.size() * sizeof(TileSlot), cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess && !gm.empty())
+      e = cudaMemcpy(gm.data(), p->d_gemms, gm.size() * sizeof(GemmParam), cudaMemcpyDeviceToHost);
+    if (cur >= 0) cudaSetDevice(cur);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy(export)");
+  }
+  if (block_ptr) std::copy(bp.begin(), bp.end(), block_ptr);
+  for (size_t s = 0; s < sl.size(); ++s) {
+    if (tile_gemm) tile_gemm[s] = (int32_t)sl[s].gemm;
+    if (tile_y) tile_y[s] = sl[s].y;
+    if (tile_x) tile_x[s] = sl[s].x;
+  }
+  if (gemm_strategy) {
+    int vi = 0;
+    for (int v = 0; v < p->table->n_versions; ++v)
+      if (p->table->versions[v] == p->tiling.version_T) vi = v;
+    for (size_t i = 0; i < gm.size(); ++i) gemm_strategy[i] = vi * p->table->n_rows + (gm[i].row & 0xFF);
+  }
+  return VB_OK;
+}
+
+extern "C" vb_status vb_plan_tiler_trace(vb_plan_t p, int32_t cap, int64_t *tlp, int32_t *version_T,
+                                         int32_t *n_rounds) {
+  if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
+  const int n = (int)p->tiling.trace.size();
+  if (n_rounds) *n_rounds = n;
+  for (int i = 0; i < n && i < cap; ++i) {
+    if (tlp) tlp[i] = p->tiling.trace[(size_t)i].tlp;
+    if (version_T) version_T[i] = p->tiling.trace[(size_t)i].version_T;
+  }
+  return VB_OK;
+}
+
+extern "C" vb_status vb_plan_destroy(vb_plan_t p) {
+  delete p;
+  return VB_OK;
+}
+
+extern "C" vb_status vb_shard_lpt(int32_t batch, const int32_t *M, const int32_t *N, const int32_t *K,
+                                  int32_t n_ranks, int32_t *rank_of) {
+  if (batch < 0 || n_ranks <= 0) return fail(VB_ERR_INVALID_ARG, "batch < 0 or n_ranks <= 0");
+  if (batch > 0 && (!M || !N || !K || !rank_of)) return fail(VB_ERR_INVALID_ARG, "null array");
+  for (int i = 0; i < batch; ++i)
+    if (M[i] < 0 || N[i] < 0 || K[i] < 0) return fail(VB_ERR_INVALID_ARG, "negative size");
+  try {
+    std::vector<int32_t> r = shard_lpt(M, N, K, batch, n_ranks);
+    std::copy(r.begin(), r.end(), rank_of);
+  } catch (...) {
+    return fail(VB_ERR_OOM, "host allocation failed");
+  }
+  return VB_OK;
+}
+
+extern "C" vb_status vb_fill_uniform_batch(vb_dtype dt, int32_t batch, const int32_t *rows, const int32_t *cols,
+                                           const int32_t *ld, void *const *ptrs, const int64_t *gemm_id,
+                                           uint64_t seed, int32_t operand, int64_t total_elems, void *stream) {
+  if (batch < 0) return fail(VB_ERR_INVALID_ARG, "batch < 0");
+  if (batch == 0) return VB_OK;
+  if (!rows || !cols || !ld || !ptrs || !gemm_id) return fail(VB_ERR_INVALID_ARG, "null array");
+  cudaError_t e = launch_fill((int)dt, batch, rows, cols, ld, ptrs, gemm_id, seed, operand, total_elems,
+                              static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? VB_OK : cuda_fail(e, "fill kernel");
+}
+
+extern "C" vb_status vb_fill_alpha_beta(int32_t batch, const int64_t *gemm_id, uint64_t seed, float *alpha,
+                                        float *beta, void *stream) {
+  if (batch < 0) return fail(VB_ERR_INVALID_ARG, "batch < 0");
+  if (batch == 0) return VB_OK;
+  if (!gemm_id || !alpha || !beta) return fail(VB_ERR_INVALID_ARG, "null array");
+  cudaError_t e = launch_alpha_beta(batch, gemm_id, seed, alpha, beta, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? VB_OK : cuda_fail(e, "alpha/beta kernel");
+}
+
+extern "C" vb_status vb_device_info(int device, int32_t *sm_count, int32_t *cc_major, int32_t *cc_minor) {
+  cudaDeviceProp prop;
+  cudaError_t e = cudaGetDeviceProperties(&prop, device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceProperties");
+  if (sm_count) *sm_count = prop.multiProcessorCount;
+  if (cc_major) *cc_major = prop.major;
+  if (cc_minor) *cc_minor = prop.minor;
+  return VB_OK;
+}
+
+extern "C" const char *vb_status_str(vb_status s) {
+  switch (s) {
+    case VB_OK: return "VB_OK";
+    case VB_ERR_INVALID_ARG: return "VB_ERR_INVALID_ARG";
+    case VB_ERR_ALIGNMENT: return "VB_ERR_ALIGNMENT";
+    case VB_ERR_UNSUPPORTED: return "VB_ERR_UNSUPPORTED";
+    case VB_ERR_OOM: return "VB_ERR_OOM";
+    case VB_ERR_CUDA: return "VB_ERR_CUDA";
+    case VB_ERR_INTERNAL: return "VB_ERR_INTERNAL";
+  }
+  return "VB_ERR_UNKNOWN";
+}
+
+extern "C" const char *vb_last_error(void) { return g_last_error.c_str(); }
+
+extern "C" const char *vb_version(void) { return "vbgemm-b200 0.1 (sm_100a)"; }

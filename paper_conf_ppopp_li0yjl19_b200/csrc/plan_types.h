@@ -1,0 +1,73 @@
+// Device-visible plan layout shared by the host C-ABI (capi.cu) and the kernels.
+//
+// The five auxiliary arrays of PAPER.md §6 (P282, Fig. 6) are packed as:
+//   block_ptr[n_blocks+1]           == Tile[]                      (CSR over tile slots)
+//   TileSlot{gemm, y, x}[n_slots]   == GEMM[], Y_Coord[], X_Coord[] (8 bytes per slot)
+//   GemmParam[batch].row            == Tiling[] (per GEMM, reading C-12)
+#pragma once
+#include <stdint.h>
+
+namespace vb {
+
+struct alignas(8) TileSlot {
+  uint32_t gemm;
+  uint16_t y;   // tile row index along M   (element origin y * BY)
+  uint16_t x;   // tile column index along N (element origin x * BX)
+};
+static_assert(sizeof(TileSlot) == 8, "TileSlot must stay 8 bytes");
+
+struct alignas(16) GemmParam {
+  int32_t M, N, K;
+  int32_t lda, ldb, ldc;
+  int32_t row;       // strategy row in the plan's table
+  int32_t kblocks;   // ceil(K / BK)
+};
+static_assert(sizeof(GemmParam) == 32, "GemmParam must stay 32 bytes");
+
+// Kernel arguments (by value).
+struct F32Args {
+  const int32_t *block_ptr;
+  const TileSlot *slots;
+  const GemmParam *gemms;
+  const float *const *A;
+  const float *const *B;
+  float *const *C;
+  const float *alpha;
+  const float *beta;
+};
+
+struct TcArgs {
+  const int32_t *block_ptr;
+  const TileSlot *slots;
+  const GemmParam *gemms;
+  const void *tmaps;        // CUtensorMap[batch][3] = {A, B, C}, 128-byte aligned
+  void *const *C;           // C pointers (direct stores of row tails that TMA cannot clip)
+  const float *alpha;
+  const float *beta;
+  int32_t *counter;         // dynamic work-list counter (reset by the prep kernel)
+  int32_t n_blocks;
+};
+
+// Tensor-core strategy geometry derived from a table row (BY, BX): TMA boxes and swizzles.
+struct TcGeom {
+  int BY, BX;
+  int b_swz;       // bytes of one swizzled B row segment (32/64/128) = box inner extent
+  int b_boxes;     // B boxes per k-block (BX / (b_swz/2))
+  int c_cols;      // C chunk width in elements (one TMA box)
+  int c_swz;       // bytes of one swizzled C row segment
+  int c_chunks;    // BX / c_cols
+};
+
+__host__ __device__ inline TcGeom tc_geom(int BY, int BX) {
+  TcGeom g;
+  g.BY = BY;
+  g.BX = BX;
+  g.b_swz = BX >= 64 ? 128 : BX * 2;
+  g.b_boxes = BX / (g.b_swz / 2);
+  g.c_cols = BX >= 64 ? 64 : BX;
+  g.c_swz = g.c_cols * 2;
+  g.c_chunks = BX / g.c_cols;
+  return g;
+}
+
+}  // namespace vb

@@ -1,0 +1,60 @@
+// Strategy tables of the product path.  The oracle keeps its own,
+// independently restated copy (oracle/plan_ref.py); the two are compared only by tests.
+#pragma once
+#include <stdint.h>
+
+namespace vb {
+
+struct StrategyRow {
+  const char *name;
+  int BY;   // C-tile rows    (along M)
+  int BX;   // C-tile columns (along N)
+  int BK;   // K step of one main-loop iteration
+};
+
+constexpr int kMaxRows = 6;
+constexpr int kMaxVersions = 2;
+
+struct TableDef {
+  int id;
+  const char *name;
+  int n_rows;
+  StrategyRow rows[kMaxRows];
+  int n_versions;
+  int versions[kMaxVersions];   // thread counts T, preferred (more TLP) first — P247
+  int64_t tlp_threshold;        // P253 / P290 (platform constant)
+  int theta;                    // P259 / P290 (platform constant)
+};
+
+// PAPER.md Table 2 (P204-214): small 16x16, medium 32x32, large 64x64, tall 128x64,
+// wide 64x128, huge 128x128; BK = 8 (P243); 256- and 128-thread versions (P181, P198).
+#define VB_TABLE2_ROWS                                                              \
+  {{"small", 16, 16, 8}, {"medium", 32, 32, 8}, {"large", 64, 64, 8},               \
+   {"tall", 128, 64, 8}, {"wide", 64, 128, 8}, {"huge", 128, 128, 8}}
+
+// V100 profile: the paper's constants (P255, P290).
+constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 128}, 65536, 256};
+
+// B200 FFMA profile (fp32): Table 2 shapes/sub-tiles (an FFMA design that still holds on
+// sm_100a), threshold re-set for 148 SMs (reading C-22, calibration is NEXT-1).
+constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 2, {256, 128}, 131072, 256};
+
+// B200 tcgen05 profile (bf16/fp16): tcgen05.mma M in {64,128}; BK = 64 = one 128-byte
+// swizzled row of bf16; one kernel version with 256 threads (8 warps).
+constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 6,
+                                   {{"s", 64, 32, 64}, {"m", 64, 64, 64}, {"t", 128, 64, 64},
+                                    {"w", 64, 128, 64}, {"l", 128, 128, 64}, {"h", 128, 256, 64}},
+                                   1, {256, 0}, 4 * 148 * 256, 512};
+
+#undef VB_TABLE2_ROWS
+
+inline const TableDef *table_by_id(int id) {
+  switch (id) {
+    case 1: return &kTableV100;
+    case 2: return &kTableB200Ffma;
+    case 3: return &kTableB200Tc;
+    default: return nullptr;
+  }
+}
+
+}  // namespace vb

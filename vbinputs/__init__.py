@@ -12,7 +12,7 @@ Generator (PAPER.md P444 only says "random matrix size an
 * element value    ``h = splitmix64(mkey + idx)``, ``idx = i*cols + j`` (LOGICAL index, so the
   leading-dimension padding never changes a value)
 * matrix entries   ``u = (h >> 40) * 2^-23 - 1``  -> uniform on [-1, 1), exact in fp32
-* alpha            ``0.5 + (h >> 40) * 2^-24``      -> [0.5, 1.5)   (operand 3, idx 0)
+* alpha            ``0.5 + (h >> 41) * 2^-23``      -> [0.5, 1.5)   (operand 3, idx 0)
 * beta             ``(h >> 40) * 2^-23 - 1``        -> [-1, 1)      (operand 4, idx 0)
 * bf16 / fp16 inputs are the fp32 draw rounded to nearest-even.
 """
@@ -113,6 +113,6 @@ def alpha_beta(seed: int, gemms, mode: str = "random"):
     al = np.empty(len(gemms), np.float32)
     be = np.empty(len(gemms), np.float32)
     for t, g in enumerate(gemms):
-        al[t] = np.float32(0.5 + float(_u24(seed, int(g), OP_ALPHA, [0])[0]) * 2.0 ** -24)
+        al[t] = np.float32(0.5 + float(_u24(seed, int(g), OP_ALPHA, [0])[0] >> 1) * 2.0 ** -23)
         be[t] = np.float32(float(_u24(seed, int(g), OP_BETA, [0])[0]) * 2.0 ** -23 - 1.0)
     return al, be
