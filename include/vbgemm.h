@@ -118,13 +118,27 @@ vb_status vb_plan_from_schedule(int device, vb_dtype dt, int32_t batch,
  *  alpha, beta  DEVICE fp32 arrays [batch].
  *  stream   cudaStream_t as void*.
  * Never allocates, never synchronises.  Enqueues at most two kernels (a descriptor
- * prep kernel for the tensor-core path, then the persistent GEMM kernel).  The caller
+ * prep kernel, then the GEMM kernel; the fp32 path needs no prep kernel).  The caller
  * keeps every buffer alive until the stream work completes.  A plan may be re-executed
  * with new pointers / alpha / beta, but not concurrently on two streams.
  * Returns VB_ERR_CUDA if a launch fails (vb_last_error() has the CUDA message).
  * ------------------------------------------------------------------------------------ */
 vb_status vb_exec_vbatched(vb_plan_t plan, const void *const *A, const void *const *B,
                            void *const *C, const float *alpha, const float *beta, void *stream);
+
+/* ------------------------------------------------------------------------------------
+ * vb_plan_bind / vb_exec_bound — vb_exec_vbatched split in two for callers that run the
+ * same buffers many times (e.g. a fixed batch in DNN training, P272):
+ *  vb_plan_bind   records the DEVICE pointer arrays A, B, C in the plan and enqueues the
+ *                 descriptor prep kernel (tensor-map address patch) on `stream`.  The arrays
+ *                 and matrices must stay valid until the last vb_exec_bound using them ends.
+ *  vb_exec_bound  enqueues only the GEMM kernel, using the last bound pointers and the
+ *                 given alpha/beta (DEVICE fp32 [batch]).  VB_ERR_INVALID_ARG if never bound.
+ * vb_exec_vbatched(...) == vb_plan_bind(...) + vb_exec_bound(...).
+ * ------------------------------------------------------------------------------------ */
+vb_status vb_plan_bind(vb_plan_t plan, const void *const *A, const void *const *B, void *const *C,
+                       void *stream);
+vb_status vb_exec_bound(vb_plan_t plan, const float *alpha, const float *beta, void *stream);
 
 /* ------------------------------------------------------------------------------------
  * vb_plan_info — sizes of the plan (any output pointer may be NULL).

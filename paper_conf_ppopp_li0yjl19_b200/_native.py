@@ -51,6 +51,8 @@ lib.vb_plan_vbatched.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int32] + [
 lib.vb_plan_from_schedule.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int32] + [_i32p] * 6 + \
     [ctypes.c_int32, _i32p, ctypes.c_int32, ctypes.c_int32, _i32p, _i32p, _i32p, _i32p, _P(_vp)]
 lib.vb_exec_vbatched.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp]
+lib.vb_plan_bind.argtypes = [_vp, _vp, _vp, _vp, _vp]
+lib.vb_exec_bound.argtypes = [_vp, _vp, _vp, _vp]
 lib.vb_plan_info.argtypes = [_vp, _i64p, _i64p, _i64p, _i32p, _i32p]
 lib.vb_plan_export.argtypes = [_vp, _i32p, _i32p, _i32p, _i32p, _i32p]
 lib.vb_plan_tiler_trace.argtypes = [_vp, ctypes.c_int32, _i64p, _i32p, _i32p]
@@ -60,7 +62,7 @@ lib.vb_fill_uniform_batch.argtypes = [ctypes.c_int, ctypes.c_int32, _vp, _vp, _v
                                       ctypes.c_int32, ctypes.c_int64, _vp]
 lib.vb_fill_alpha_beta.argtypes = [ctypes.c_int32, _vp, ctypes.c_uint64, _vp, _vp, _vp]
 lib.vb_device_info.argtypes = [ctypes.c_int, _i32p, _i32p, _i32p]
-for _f in ("vb_plan_vbatched", "vb_plan_from_schedule", "vb_exec_vbatched", "vb_plan_info", "vb_plan_export",
+for _f in ("vb_plan_vbatched", "vb_plan_from_schedule", "vb_exec_vbatched", "vb_plan_bind", "vb_exec_bound", "vb_plan_info", "vb_plan_export",
            "vb_plan_tiler_trace", "vb_plan_destroy", "vb_shard_lpt", "vb_fill_uniform_batch", "vb_fill_alpha_beta",
            "vb_device_info"):
     getattr(lib, _f).restype = ctypes.c_int
@@ -142,6 +144,12 @@ class Plan:
         """All arguments are raw DEVICE addresses (ints); stream is a cudaStream_t as int."""
         check(lib.vb_exec_vbatched(self.handle, _vp(A_ptrs), _vp(B_ptrs), _vp(C_ptrs), _vp(alpha), _vp(beta),
                                    _vp(stream)))
+
+    def bind(self, A_ptrs: int, B_ptrs: int, C_ptrs: int, stream: int = 0) -> None:
+        check(lib.vb_plan_bind(self.handle, _vp(A_ptrs), _vp(B_ptrs), _vp(C_ptrs), _vp(stream)))
+
+    def exec_bound(self, alpha: int, beta: int, stream: int = 0) -> None:
+        check(lib.vb_exec_bound(self.handle, _vp(alpha), _vp(beta), _vp(stream)))
 
 
 def plan_vbatched(M, N, K, lda, ldb, ldc, dtype: str = "bf16", policy: int = VB_BATCH_THRESHOLD,

@@ -123,6 +123,15 @@ class DeviceBatch:
                                 theta=theta)
 
     def run(self, plan: nv.Plan, stream=None) -> None:
+        """vb_exec_vbatched: bind this batch's pointers and run (two launches on the tc path)."""
         s = torch.cuda.current_stream(self.device) if stream is None else stream
         plan.exec(self.pA.data_ptr(), self.pB.data_ptr(), self.pC.data_ptr(), self.alpha.data_ptr(),
                   self.beta.data_ptr(), s.cuda_stream)
+
+    def bind(self, plan: nv.Plan, stream=None) -> None:
+        s = torch.cuda.current_stream(self.device) if stream is None else stream
+        plan.bind(self.pA.data_ptr(), self.pB.data_ptr(), self.pC.data_ptr(), s.cuda_stream)
+
+    def run_bound(self, plan: nv.Plan, stream=None) -> None:
+        s = torch.cuda.current_stream(self.device) if stream is None else stream
+        plan.exec_bound(self.alpha.data_ptr(), self.beta.data_ptr(), s.cuda_stream)

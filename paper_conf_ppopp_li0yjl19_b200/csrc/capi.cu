@@ -20,8 +20,9 @@
 
 namespace vb {
 cudaError_t launch_f32(const F32Args &args, int n_blocks, int version_T, cudaStream_t stream);
-cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, uint8_t *tmaps, const void *const *A,
-                      const void *const *B, void *const *C, const GemmParam *gemms, int batch, cudaStream_t stream);
+cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
+                           const GemmParam *gemms, int batch, int32_t *counter, cudaStream_t stream);
+cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, cudaStream_t stream);
 cudaError_t tc_configure();
 size_t tc_smem_bytes();
 cudaError_t launch_fill(int dt, int batch, const int32_t *rows, const int32_t *cols, const int32_t *ld,
@@ -65,8 +66,11 @@ struct vb_plan {
   TileSlot *d_slots = nullptr;
   GemmParam *d_gemms = nullptr;
   uint8_t *d_tmaps = nullptr;
-  int32_t *d_counter = nullptr;
+  int32_t *d_counter = nullptr;     // [0] work-list counter, [1] finished-CTA counter
   int sm_count = 0;
+  const void *const *bound_A = nullptr;   // last vb_plan_bind
+  const void *const *bound_B = nullptr;
+  void *const *bound_C = nullptr;
   ~vb_plan() {
     if (d_ws) {
       int prev = 0;
@@ -364,33 +368,67 @@ extern "C" vb_status vb_plan_from_schedule(int device, vb_dtype dt, int32_t batc
   }
 }
 
-extern "C" vb_status vb_exec_vbatched(vb_plan_t p, const void *const *A, const void *const *B, void *const *C,
-                                      const float *alpha, const float *beta, void *stream) {
+struct DeviceGuard {
+  int prev = -1;
+  cudaError_t err = cudaSuccess;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) err = cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+extern "C" vb_status vb_plan_bind(vb_plan_t p, const void *const *A, const void *const *B, void *const *C,
+                                  void *stream) {
+  if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
+  if (p->device < 0) return fail(VB_ERR_UNSUPPORTED, "host-only plan cannot be executed");
+  if (p->batch > 0 && (!A || !B || !C)) return fail(VB_ERR_INVALID_ARG, "null pointer array");
+  p->bound_A = A;
+  p->bound_B = B;
+  p->bound_C = C;
+  if (p->batch == 0 || p->dt == VB_F32) return VB_OK;
+  DeviceGuard g(p->device);
+  if (g.err != cudaSuccess) return cuda_fail(g.err, "cudaSetDevice");
+  cudaError_t e = launch_tc_prep(p->d_tmaps, A, B, C, p->d_gemms, p->batch, p->d_counter,
+                                 static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? VB_OK : cuda_fail(e, "prep kernel launch");
+}
+
+extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float *beta, void *stream) {
   if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
   if (p->device < 0) return fail(VB_ERR_UNSUPPORTED, "host-only plan cannot be executed");
   if (p->batch == 0) return VB_OK;
-  if (!A || !B || !C || !alpha || !beta) return fail(VB_ERR_INVALID_ARG, "null argument array");
-  int cur = -1;
-  cudaGetDevice(&cur);
-  if (cur != p->device) {
-    cudaError_t e = cudaSetDevice(p->device);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
-  }
+  if (!p->bound_A) return fail(VB_ERR_INVALID_ARG, "plan was never bound (vb_plan_bind)");
+  if (!alpha || !beta) return fail(VB_ERR_INVALID_ARG, "null alpha/beta");
+  DeviceGuard g(p->device);
+  if (g.err != cudaSuccess) return cuda_fail(g.err, "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   const int n_blocks = (int)p->block_ptr.size() - 1;
   cudaError_t e;
   if (p->dt == VB_F32) {
-    F32Args a{p->d_block_ptr, p->d_slots, p->d_gemms, reinterpret_cast<const float *const *>(A),
-              reinterpret_cast<const float *const *>(B), reinterpret_cast<float *const *>(C), alpha, beta};
+    F32Args a{p->d_block_ptr, p->d_slots, p->d_gemms, reinterpret_cast<const float *const *>(p->bound_A),
+              reinterpret_cast<const float *const *>(p->bound_B), reinterpret_cast<float *const *>(p->bound_C),
+              alpha, beta};
     e = launch_f32(a, n_blocks, p->tiling.version_T, s);
   } else {
-    TcArgs a{p->d_block_ptr, p->d_slots, p->d_gemms, p->d_tmaps, C, alpha, beta, p->d_counter, n_blocks};
-    const int grid = std::min(n_blocks, p->sm_count);
-    e = launch_tc(a, grid, p->dt == VB_BF16, p->d_tmaps, A, B, C, p->d_gemms, p->batch, s);
+    TcArgs a{p->d_block_ptr, p->d_slots, p->d_gemms, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_blocks};
+    e = launch_tc(a, std::min(n_blocks, p->sm_count), p->dt == VB_BF16, s);
   }
-  if (cur != p->device && cur >= 0) cudaSetDevice(cur);
-  if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
-  return VB_OK;
+  return e == cudaSuccess ? VB_OK : cuda_fail(e, "kernel launch");
+}
+
+extern "C" vb_status vb_exec_vbatched(vb_plan_t p, const void *const *A, const void *const *B, void *const *C,
+                                      const float *alpha, const float *beta, void *stream) {
+  if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
+  if (p->device >= 0 && p->batch > 0 && (!A || !B || !C || !alpha || !beta))
+    return fail(VB_ERR_INVALID_ARG, "null argument array");
+  vb_status st = vb_plan_bind(p, A, B, C, stream);
+  if (st != VB_OK) return st;
+  return vb_exec_bound(p, alpha, beta, stream);
 }
 
 extern "C" vb_status vb_plan_info(vb_plan_t p, int64_t *n_tiles, int64_t *n_blocks, int64_t *workspace_bytes,
@@ -402,7 +440,7 @@ extern "C" vb_status vb_plan_info(vb_plan_t p, int64_t *n_tiles, int64_t *n_bloc
   if (version_T) *version_T = p->tiling.version_T;
   if (launches_per_exec) {
     const bool any = p->block_ptr.size() > 1;
-    *launches_per_exec = p->batch == 0 ? 0 : (p->dt == VB_F32 ? (any ? 1 : 0) : (any ? 2 : 1));
+    *launches_per_exec = p->batch == 0 ? 0 : (p->dt == VB_F32 ? (any ? 1 : 0) : (any ? 2 : 1));  // prep + GEMM
   }
   return VB_OK;
 }

@@ -372,6 +372,16 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   __syncthreads();
   ptx::tc_fence_after();
   if (warp == 2) ptx::tmem_dealloc(tmem_base, kTmemCols);
+  // The last CTA to finish resets the work-list counter, so back-to-back launches of the
+  // same bound plan need no reset kernel.  Every CTA fetched past n_blocks before getting here.
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(&p.counter[1], 1) == (int)gridDim.x - 1) {
+      atomicExch(&p.counter[0], 0);
+      atomicExch(&p.counter[1], 0);
+      __threadfence();
+    }
+  }
 }
 
 // Exec-time prep: patch the global address of every per-GEMM tensor map (A, B, C) with the
@@ -379,7 +389,10 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
                            const GemmParam *gemms, int batch, int32_t *counter) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i == 0) *counter = 0;
+  if (i == 0) {
+    counter[0] = 0;
+    counter[1] = 0;
+  }
   if (i >= batch * 3) return;
   const int g = i / 3, w = i % 3;
   const GemmParam gp = gemms[g];
@@ -402,13 +415,15 @@ cudaError_t tc_configure() {
                               (int)tck::kSmemBytes);
 }
 
-cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, uint8_t *tmaps, const void *const *A,
-                      const void *const *B, void *const *C, const GemmParam *gemms, int batch, cudaStream_t stream) {
+cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
+                           const GemmParam *gemms, int batch, int32_t *counter, cudaStream_t stream) {
   const int n = batch * 3;
-  tck::vb_tc_prep<<<(n + 255) / 256 > 0 ? (n + 255) / 256 : 1, 256, 0, stream>>>(tmaps, A, B, C, gemms, batch,
-                                                                                  args.counter);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess || grid <= 0) return e;
+  tck::vb_tc_prep<<<n > 0 ? (n + 255) / 256 : 1, 256, 0, stream>>>(tmaps, A, B, C, gemms, batch, counter);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, cudaStream_t stream) {
+  if (grid <= 0) return cudaSuccess;
   if (bf16)
     tck::vb_tc_kernel<1><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
   else

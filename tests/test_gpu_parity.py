@@ -223,3 +223,23 @@ def test_bitwise_deterministic_and_reexecutable(dtype):
     # beta close to -1 makes C2 = (1+beta)*alpha*AB + beta^2*C0 cancel, so the normwise
     # measure is not meaningful here; check the elementwise forward-error bound instead
     check_bound(db, range(len(M)), SEED, "random", c_old=c1)
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+def test_bind_then_exec_bound_repeatedly(dtype):
+    # exec_bound launches only the GEMM kernel; the kernel resets its own work counter, so
+    # back-to-back launches must each process the whole batch
+    M, N, K = vbinputs.config_sizes("C2")
+    M, N, K = M[:48], N[:48], K[:48]
+    db = DeviceBatch(M, N, K, dtype)
+    db.fill(SEED)
+    plan = db.plan()
+    db.bind(plan)
+    c_prev = None
+    for it in range(3):
+        c_prev = [to_f64(db.c(g)).copy() for g in range(len(M))]
+        db.run_bound(plan)
+        torch.cuda.synchronize()
+        check_bound(db, range(len(M)), SEED, "random", c_old=c_prev)
+    with pytest.raises(vb.VbError):
+        db.plan().exec_bound(db.alpha.data_ptr(), db.beta.data_ptr(), 0)   # never bound

@@ -73,3 +73,11 @@ def test_config_recipes():
 def test_padded_ld():
     assert list(vi.padded_ld([1, 8, 9, 17], "bf16")) == [8, 8, 16, 24]
     assert list(vi.padded_ld([1, 4, 5], "f32")) == [4, 4, 8]
+
+
+def test_c_generator_matches_numpy_reference():
+    for dtype in ("f32", "bf16", "f16"):
+        for (g, op, r, c) in ((0, 0, 17, 33), (70000, 2, 64, 129), (5, 1, 1, 1)):
+            ref = vi.matrix(42, g, op, r, c, dtype)[1]
+            fast = vi.matrix_f64_fast(42, g, op, r, c, dtype)
+            assert np.array_equal(ref, fast), (dtype, g, op)

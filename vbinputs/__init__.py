@@ -105,6 +105,38 @@ def matrix(seed: int, gemm: int, operand: int, rows: int, cols: int, dtype: str)
     return quantize(uniform_f32(seed, gemm, operand, rows, cols), dtype)
 
 
+_gen_lib = None
+
+
+def _gen():
+    """ctypes handle of the C implementation of the same generator (built on first use)."""
+    global _gen_lib
+    if _gen_lib is None:
+        import ctypes
+        import os
+        import subprocess
+        here = os.path.dirname(os.path.abspath(__file__))
+        src, so = os.path.join(here, "_gen.c"), os.path.join(here, "_gen.so")
+        if not os.path.exists(so) or os.path.getmtime(so) < os.path.getmtime(src):
+            tmp = so + f".tmp{os.getpid()}"
+            subprocess.check_call(["gcc", "-O2", "-fopenmp", "-ffp-contract=off", "-fPIC", "-shared", "-o", tmp, src])
+            os.replace(tmp, so)
+        lib = ctypes.CDLL(so)
+        lib.vbgen_fill_f64.argtypes = [ctypes.c_uint64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.c_void_p]
+        lib.vbgen_fill_f64.restype = None
+        _gen_lib = lib
+    return _gen_lib
+
+
+def matrix_f64_fast(seed: int, gemm: int, operand: int, rows: int, cols: int, dtype: str) -> np.ndarray:
+    """Exact fp64 values of ``matrix(...)[1]`` from the C generator (multi-threaded)."""
+    out = np.empty((rows, cols), np.float64)
+    if out.size:
+        _gen().vbgen_fill_f64(matrix_key(seed, gemm, operand), rows, cols, {"f32": 0, "bf16": 1, "f16": 2}[dtype],
+                              out.ctypes.data)
+    return out
+
+
 def alpha_beta(seed: int, gemms, mode: str = "random"):
     """Per-GEMM fp32 alpha/beta. mode 'random' (alpha in [0.5,1.5), beta in [-1,1)) or 'conv' (1, 0)."""
     gemms = np.asarray(gemms, dtype=np.int64)
