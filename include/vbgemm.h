@@ -57,8 +57,9 @@ typedef enum { VB_BATCH_THRESHOLD = 0, VB_BATCH_BINARY = 1, VB_BATCH_NONE = 2 } 
  *  VB_TABLE_V100        PAPER.md Table 2 (P204-214) with the V100 constants (P290):
  *                       TLP threshold 65536, theta 256, versions T = 256 / 128.
  *  VB_TABLE_B200_FFMA   Table 2 shapes for the fp32 FFMA kernel, B200 constants.
- *  VB_TABLE_B200_TC     tcgen05 table (bf16/fp16): 64x32, 64x64, 128x64, 64x128,
- *                       128x128, 128x256 C tiles, BK = 64, T = 256.
+ *  VB_TABLE_B200_TC     tcgen05 table (bf16/fp16): 64x32, 128x32, 64x64, 128x64, 64x128,
+ *                       128x128, 64x256, 128x256 C tiles, BK = 64, T = 256; availability
+ *                       tested against max(M, 64) x max(N, 32) (the 64-row MMA floor).
  *  VB_TABLE_DEFAULT     B200_FFMA for VB_F32, B200_TC for VB_BF16 / VB_F16. */
 typedef enum {
   VB_TABLE_DEFAULT = 0, VB_TABLE_V100 = 1, VB_TABLE_B200_FFMA = 2, VB_TABLE_B200_TC = 3

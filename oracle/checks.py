@@ -93,5 +93,6 @@ def check_plan_invariants(p: Plan, Ms, Ns, Ks, policy: int, theta: int) -> None:
         assert all(pos[b] >= pos[a] for a, b in zip(r0, r1))
     for g, (m, n) in enumerate(zip(Ms, Ns)):
         s = p.table.rows[p.tiling.rows[g]]
-        fits_any = any(q.BY <= m and q.BX <= n for q in p.table.rows)
-        assert (s.BY <= m and s.BX <= n) or (not fits_any and p.tiling.rows[g] == p.table.order()[0])
+        mf, nf = max(m, p.table.min_BY), max(n, p.table.min_BX)
+        fits_any = any(q.BY <= mf and q.BX <= nf for q in p.table.rows)
+        assert (s.BY <= mf and s.BX <= nf) or (not fits_any and p.tiling.rows[g] == p.table.order()[0])

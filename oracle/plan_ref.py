@@ -31,6 +31,8 @@ class Table:
     versions: Tuple[int, ...]            # thread counts T, first = preferred (more TLP)
     tlp_threshold: int                   # default TLP threshold (P253, P290)
     theta: int                           # default batching threshold θ (P259, P290)
+    min_BY: int = 0                      # availability floor (reading C-1b); 0 = the paper's rule
+    min_BX: int = 0
 
     def order(self) -> List[int]:
         """Priority order: smaller tile first (P249); ties by table row (reading C-3)."""
@@ -53,12 +55,15 @@ V100 = Table("v100_table2", (
 B200_F32 = Table("b200_ffma", V100.rows, versions=(256, 128), tlp_threshold=131072, theta=256)
 
 # B200 tcgen05 (bf16/fp16) profile: C-tile shapes sized for tcgen05.mma
-# (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16).  One kernel "version" with
-# T = 256 threads (8 warps), so the paper's version switch is a no-op for this table.
+# (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16), plus the skinny shapes
+# 128x32 and 64x256.  One kernel "version" with T = 256 threads (8 warps).  Availability
+# floor (C-1b): a GEMM shorter than 64 rows still occupies a 64-row MMA, so strategies are
+# tested against max(M, 64) and max(N, 32).
 B200_TC = Table("b200_tcgen05", (
-    Strategy("s", 64, 32, 64), Strategy("m", 64, 64, 64), Strategy("t", 128, 64, 64),
-    Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("h", 128, 256, 64)),
-    versions=(256,), tlp_threshold=4 * 148 * 256, theta=512)
+    Strategy("s", 64, 32, 64), Strategy("n", 128, 32, 64), Strategy("m", 64, 64, 64), Strategy("t", 128, 64, 64),
+    Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("x", 64, 256, 64),
+    Strategy("h", 128, 256, 64)),
+    versions=(256,), tlp_threshold=4 * 148 * 256, theta=512, min_BY=64, min_BX=32)
 
 TABLES = {1: V100, 2: B200_F32, 3: B200_TC}
 
@@ -88,35 +93,41 @@ class TilingResult:
 def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None) -> TilingResult:
     """The three steps and two exceptions of P249–253.
 
-    1. Per GEMM, a priority queue of the strategies with BY <= M and BX <= N (C-1),
+    1. Per GEMM, a priority queue of the strategies with BY <= M and BX <= N (C-1; the
+       B200 tcgen05 table compares against max(M, 64) and max(N, 32), C-1b),
        smallest first (P249); if none fits, the smallest strategy alone (C-4).
     2. Take one strategy per GEMM: pop, or top if only one is left (exception 1, C-2);
        TLP by Eq. 1 with the current version T.
     3. If TLP > threshold (strict, C-6) repeat step 2; otherwise this is the solution.
        Exception 2 (C-7): if step 2 is to be repeated while every queue holds a single
-       strategy, switch to the second version (128 threads) and repeat step 2 once more;
-       if no further version exists, stop with the current solution.
+       strategy, switch to the next version (128 threads) and repeat step 2.  With no
+       further version, step 2 is still repeated once if this round popped (so the last,
+       largest strategy of each queue is evaluated); if this round already took the top of
+       every queue there is nothing larger to try and the current solution stands.
     """
     thr = table.tlp_threshold if threshold is None else threshold
     order = table.order()
     queues = []
     for M, N in zip(Ms, Ns):
-        q = [r for r in order if table.rows[r].BY <= M and table.rows[r].BX <= N]
+        mf, nf = max(M, table.min_BY), max(N, table.min_BX)           # C-1b (0 for the paper's tables)
+        q = [r for r in order if table.rows[r].BY <= mf and table.rows[r].BX <= nf]
         queues.append(q if q else [order[0]])
     vi = 0
     T = table.versions[vi]
     trace = []
     while True:
+        single_before = all(len(q) == 1 for q in queues)
         cur = [q.pop(0) if len(q) > 1 else q[0] for q in queues]       # step 2
         t = tlp(Ms, Ns, cur, table, T)
         trace.append((list(cur), T, t))
         if t <= thr:                                                   # step 3
             return TilingResult(cur, T, trace)
         if all(len(q) == 1 for q in queues):                           # exception 2
-            if vi + 1 >= len(table.versions):
+            if vi + 1 < len(table.versions):
+                vi += 1
+                T = table.versions[vi]
+            elif single_before:
                 return TilingResult(cur, T, trace)
-            vi += 1
-            T = table.versions[vi]
 
 
 # ----------------------------------------------------------------------------------------

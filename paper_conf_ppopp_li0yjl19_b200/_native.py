@@ -12,7 +12,8 @@ import re
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libvbgemm.so")
+# VB_LIB selects an alternative build of the same library (e.g. libvbgemm_trace.so).
+LIB_PATH = os.environ.get("VB_LIB") or os.path.join(HERE, "libvbgemm.so")
 HEADER = os.path.join(os.path.dirname(HERE), "include", "vbgemm.h")
 
 VB_OK, VB_ERR_INVALID_ARG, VB_ERR_ALIGNMENT, VB_ERR_UNSUPPORTED, VB_ERR_OOM, VB_ERR_CUDA, VB_ERR_INTERNAL = range(7)

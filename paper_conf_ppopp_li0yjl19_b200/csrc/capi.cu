@@ -35,6 +35,11 @@ cudaError_t launch_alpha_beta(int batch, const int64_t *gemm_id, uint64_t seed, 
 using namespace vb;
 
 static thread_local std::string g_last_error;
+static long long *g_trace = nullptr;   // VB_TRACE builds: device buffer for per-role wait cycles
+
+// Diagnostic hook (not in vbgemm.h): device buffer that a -DVB_TRACE build of the
+// tensor-core kernel accumulates per-role wait cycles into; nullptr disables.
+extern "C" void vb_debug_set_trace(long long *device_buf) { g_trace = device_buf; }
 
 static vb_status fail(vb_status s, const char *fmt, ...) {
   char buf[512];
@@ -65,6 +70,8 @@ struct vb_plan {
   int32_t *d_block_ptr = nullptr;
   TileSlot *d_slots = nullptr;
   GemmParam *d_gemms = nullptr;
+  TileDesc *d_tiles = nullptr;      // tensor-core path: one record per slot
+  std::vector<TileDesc> tiles;
   uint8_t *d_tmaps = nullptr;
   int32_t *d_counter = nullptr;     // [0] work-list counter, [1] finished-CTA counter
   int sm_count = 0;
@@ -172,6 +179,8 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   off = align_up(off + std::max<size_t>(p->slots.size(), 1) * sizeof(TileSlot), 256);
   const size_t o_gp = off;
   off = align_up(off + std::max<size_t>(p->gemms.size(), 1) * sizeof(GemmParam), 256);
+  const size_t o_td = off;
+  if (tc) off = align_up(off + std::max<size_t>(p->tiles.size(), 1) * sizeof(TileDesc), 256);
   const size_t o_ct = off;
   off = align_up(off + 256, 256);
   const size_t o_tm = off;
@@ -187,12 +196,14 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   p->d_slots = reinterpret_cast<TileSlot *>(base + o_sl);
   p->d_gemms = reinterpret_cast<GemmParam *>(base + o_gp);
   p->d_counter = reinterpret_cast<int32_t *>(base + o_ct);
+  p->d_tiles = tc ? reinterpret_cast<TileDesc *>(base + o_td) : nullptr;
   p->d_tmaps = tc ? base + o_tm : nullptr;
 
   std::vector<uint8_t> host(p->ws_bytes, 0);
   memcpy(host.data() + o_bp, p->block_ptr.data(), p->block_ptr.size() * sizeof(int32_t));
   if (!p->slots.empty()) memcpy(host.data() + o_sl, p->slots.data(), p->slots.size() * sizeof(TileSlot));
   if (!p->gemms.empty()) memcpy(host.data() + o_gp, p->gemms.data(), p->gemms.size() * sizeof(GemmParam));
+  if (tc && !p->tiles.empty()) memcpy(host.data() + o_td, p->tiles.data(), p->tiles.size() * sizeof(TileDesc));
   if (tc) {
     e = tc_configure();
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(tc kernel smem)");
@@ -211,8 +222,9 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
                        (uint32_t)(g.b_swz / 2), 64, g.b_swz);
         if (st != VB_OK) return st;
       }
+      // C box = one epilogue warp's sub-box: c_cols x BY/4 rows
       st = encode_2d(&maps[3 * i + 2], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)M[i], (uint64_t)ldc[i],
-                     (uint32_t)g.c_cols, (uint32_t)s.BY, g.c_swz);
+                     (uint32_t)g.c_cols, (uint32_t)(s.BY / 4), g.c_swz);
       if (st != VB_OK) return st;
     }
   }
@@ -244,6 +256,28 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
     g.ldc = ldc[i];
     g.row = p->tiling.row[i] | (s.BY << 8) | (s.BX << 16);
     g.kblocks = (int32_t)cdiv64(K[i], s.BK);
+  }
+  if (p->dt != VB_F32) {
+    p->tiles.resize(p->slots.size());
+    for (size_t k = 0; k < p->slots.size(); ++k) {
+      const TileSlot &ts = p->slots[k];
+      const GemmParam &g = p->gemms[ts.gemm];
+      const StrategyRow &s = p->table->rows[p->tiling.row[ts.gemm]];
+      const TcGeom geo = tc_geom(s.BY, s.BX);
+      TileDesc &d = p->tiles[k];
+      d.gemm = (int32_t)ts.gemm;
+      d.m0 = ts.y * s.BY;
+      d.n0 = ts.x * s.BX;
+      d.kblocks = g.kblocks;
+      d.M = g.M;
+      d.N = g.N;
+      d.ldc = g.ldc;
+      d.geo = (uint16_t)((s.BY / 16) | ((s.BX / 16) << 8));
+      // last C chunk of this tile ends inside a 16-byte granule of the row -> direct stores
+      const int last_chunk_end = d.n0 + s.BX;
+      d.flags = (uint16_t)(((g.N & 7) != 0 && last_chunk_end > g.N && d.n0 < g.N) ? 1 : 0);
+      (void)geo;
+    }
   }
   if (p->device >= 0) return upload(p, M, N, K, lda, ldb, ldc);
   return VB_OK;
@@ -415,7 +449,7 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
               alpha, beta};
     e = launch_f32(a, n_blocks, p->tiling.version_T, s);
   } else {
-    TcArgs a{p->d_block_ptr, p->d_slots, p->d_gemms, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_blocks};
+    TcArgs a{p->d_block_ptr, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_blocks, g_trace};
     e = launch_tc(a, std::min(n_blocks, p->sm_count), p->dt == VB_BF16, s);
   }
   return e == cudaSuccess ? VB_OK : cuda_fail(e, "kernel launch");
@@ -456,8 +490,16 @@ extern "C" vb_status vb_plan_export(vb_plan_t p, int32_t *block_ptr, int32_t *ti
     cudaGetDevice(&cur);
     cudaSetDevice(p->device);
     cudaError_t e = cudaMemcpy(bp.data(), p->d_block_ptr, bp.size() * sizeof(int32_t), cudaMemcpyDeviceToHost);
-    if (e == cudaSuccess && !sl.empty())
+    if (e == cudaSuccess && !sl.empty() && p->d_tiles) {   // tensor-core kernel walks TileDesc[]
+      std::vector<TileDesc> td(sl.size());
+      e = cudaMemcpy(td.data(), p->d_tiles, td.size() * sizeof(TileDesc), cudaMemcpyDeviceToHost);
+      for (size_t k = 0; k < td.size() && e == cudaSuccess; ++k) {
+        const int BY = (td[k].geo & 0xFF) * 16, BX = (td[k].geo >> 8) * 16;
+        sl[k] = TileSlot{(uint32_t)td[k].gemm, (uint16_t)(td[k].m0 / BY), (uint16_t)(td[k].n0 / BX)};
+      }
+    } else if (e == cudaSuccess && !sl.empty()) {
       e = cudaMemcpy(sl.data(), p->d_slots, sl.size() * sizeof(TileSlot), cudaMemcpyDeviceToHost);
+    }
     if (e == cudaSuccess && !gm.empty())
       e = cudaMemcpy(gm.data(), p->d_gemms, gm.size() * sizeof(GemmParam), cudaMemcpyDeviceToHost);
     if (cur >= 0) cudaSetDevice(cur);

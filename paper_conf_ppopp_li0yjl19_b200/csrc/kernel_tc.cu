@@ -3,21 +3,23 @@
 // tensor-core MMA accumulating in TMEM.
 //
 // One CTA per SM (grid = min(Block_NUM, #SMs)), 8 warps:
-//   warp 0      scheduler + A/B producer: atomically takes the next block (work list) b,
-//               publishes it in a 4-deep smem ring, then streams every tile of b through a
-//               3-stage ring of (A: BY x 64, B: 64 x BX) bf16 k-blocks with TMA.
-//   warp 1      MMA issuer: one thread issues tcgen05.mma (M = BY, N = BX, K = 16) into one
-//               of two TMEM accumulators (2 x 256 fp32 columns), commits stage releases and
-//               "accumulator full" to mbarriers.
-//   warp 2      TMEM allocator (512 columns).
-//   warp 3      C producer: TMA-loads C_old chunks (BY x 64) into a 4-slot smem ring when
+//   warp 0      scheduler: claims the next block (work list) with an atomic (one block
+//               ahead), loads its tile descriptors (one 32-byte record per tile, lanes in
+//               parallel) and alpha/beta, and publishes them in a 32-entry smem tile ring.
+//   warp 1      A/B producer: streams each tile's k-blocks (A: BY x 64, B: 64 x BX) with TMA
+//               into a PAGED ring (18 pages of 8 KB): a k-block takes only the pages it needs
+//               (2 for a 64x32 tile, 6 for 128x256), so small tiles keep up to 9 k-blocks in
+//               flight — the paper's ILP concern for small K (P151, P259) mapped to TMA depth.
+//   warp 2      TMEM allocator + MMA issuer: one thread issues tcgen05.mma (M = BY, N = BX,
+//               K = 16) into one of two 256-column fp32 accumulators.
+//   warp 3      C producer: TMA-loads C_old chunks (BY x 64) into a 4-slot ring when
 //               beta != 0 (C is never read when beta == 0, reading C-16).
-//   warps 4-7   epilogue: tcgen05.ld the accumulator (warp w owns TMEM lanes 32*(w%4)..),
-//               C = alpha*acc + beta*C_old in fp32, round-to-nearest-even to bf16/fp16,
-//               write back into the swizzled smem chunk and TMA-store it (OOB clipped).
-// The Fig. 2 double buffering (P147) becomes the TMA/mbarrier rings; the paper's "unified
-// thread structure" (P181) becomes a runtime MMA instruction descriptor per tile, so one
-// kernel serves every strategy of the table.
+//   warps 4-7   epilogue: tcgen05.ld (warp w owns TMEM lanes 32*(w%4)..), C = alpha*acc +
+//               beta*C_old in fp32, RNE to bf16/fp16, write back into the swizzled smem chunk,
+//               TMA store (completion deferred by one chunk); the accumulator is released
+//               to the MMA warp as soon as its last columns are in registers.
+// The paper's "unified thread structure" (P181) becomes a runtime MMA instruction descriptor
+// per tile, so one kernel serves every strategy of the table.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
@@ -30,36 +32,68 @@
 namespace vb {
 namespace tck {
 
-constexpr int kThreads = 256;
+constexpr int kThreads = 384;              // 4 role warps + 8 epilogue warps
 constexpr int kBK = 64;                    // bf16 elements per k-block = one 128-B swizzle row
-constexpr int kStages = 3;
-constexpr int kABytes = 128 * kBK * 2;     // 16 KB (largest BY)
-constexpr int kStageBytes = kABytes + 256 * kBK * 2;   // + 32 KB (largest BX)
+constexpr int kPageBytes = 8192;
+constexpr int kPages = 18;                 // 144 KB of A/B staging
+constexpr int kSlots = 16;                 // k-blocks in flight (bounded by pages anyway)
 constexpr int kCSlots = 4;
 constexpr int kCSlotBytes = 128 * 128;     // BY rows x 128 B
-constexpr int kSched = 4;
+constexpr int kRing = 32;                  // tile-descriptor ring entries
+constexpr int kKbAhead = 24;               // scheduler lookahead budget in k-blocks (L2 locality)
 constexpr int kTmemCols = 512;
 constexpr int kAccCols = 256;
-constexpr int kEpiThreads = 128;
-constexpr uint32_t kSchedConsumers = 1 + 1 + 4;   // MMA thread, C producer, 4 epilogue warps
+constexpr int kEpiWarps = 8;               // two per TMEM lane quarter, splitting each chunk's columns
+constexpr uint32_t kRingConsumers = 1 + 1 + 1 + kEpiWarps;   // producer, MMA, C producer, epilogue warps
 
-struct Bars {
-  uint64_t full[kStages], empty[kStages];
+struct TileInfo {          // one tile ring entry (48 bytes)
+  TileDesc d;
+  float alpha, beta;
+  int32_t pad[2];
+};
+static_assert(sizeof(TileInfo) == 48, "TileInfo size");
+
+struct Shared {
+  uint64_t full[kSlots], empty[kSlots];
   uint64_t tfull[2], tempty[2];
   uint64_t cfull[kCSlots], cempty[kCSlots];
-  uint64_t sfull[kSched], sempty[kSched];
-  int32_t sched[kSched];
+  uint64_t rfull[kRing], rempty[kRing];
+  int32_t slot_page[kSlots];
+  int32_t slot_pages[kSlots];   // producer-private: pages charged to each k-block in flight
   uint32_t tmem_base;
+  volatile uint32_t prod_kb;    // k-blocks (>= 1 per tile) the A/B producer has finished issuing
+  TileInfo ring[kRing];
 };
 
-constexpr size_t kSmemBytes = 1024 /*align slack*/ + (size_t)kStages * kStageBytes + (size_t)kCSlots * kCSlotBytes +
-                              ((sizeof(Bars) + 127) / 128) * 128;
+constexpr size_t kSmemBytes = 1024 /*align slack*/ + (size_t)kPages * kPageBytes + (size_t)kCSlots * kCSlotBytes +
+                              ((sizeof(Shared) + 127) / 128) * 128;
 
-__device__ __forceinline__ int row_BY(int packed) { return (packed >> 8) & 0xFF; }
-__device__ __forceinline__ int row_BX(int packed) { return packed >> 16; }
+// Opt-in cycle accounting (build with -DVB_TRACE): per-CTA cycles each role spends waiting
+// on each barrier, accumulated into TcArgs::trace[kTraceSlots] (unused in product builds).
+enum TraceSlot {
+  T_SCHED_REMPTY, T_SCHED_BUDGET, T_PROD_RFULL, T_PROD_EMPTY, T_MMA_RFULL, T_MMA_TEMPTY, T_MMA_FULL,
+  T_CPROD_RFULL, T_CPROD_CEMPTY, T_EPI_RFULL, T_EPI_TFULL, T_EPI_CFULL, T_EPI_STORE, T_EPI_TMEM, T_EPI_MATH,
+  T_TOTAL, T_TILES, kTraceSlots
+};
+#ifdef VB_TRACE
+#define VB_T0() const long long _vbt0 = clock64()
+#define VB_TADD(slot) tr[slot] += clock64() - _vbt0
+#define VB_TWAIT(slot, stmt) \
+  do {                       \
+    VB_T0();                 \
+    stmt;                    \
+    VB_TADD(slot);           \
+  } while (0)
+#else
+#define VB_T0()
+#define VB_TADD(slot)
+#define VB_TWAIT(slot, stmt) stmt
+#endif
 
-template <typename Ring>
-__device__ __forceinline__ void advance(Ring &idx, uint32_t &phase, int n) {
+__device__ __forceinline__ int geo_BY(uint16_t g) { return (g & 0xFF) * 16; }
+__device__ __forceinline__ int geo_BX(uint16_t g) { return (g >> 8) * 16; }
+
+__device__ __forceinline__ void advance(int &idx, uint32_t &phase, int n) {
   if (++idx == n) {
     idx = 0;
     phase ^= 1u;
@@ -72,17 +106,13 @@ __device__ __forceinline__ void unpack8(uint4 w, float (&f)[8]) {
   const uint32_t u[4] = {w.x, w.y, w.z, w.w};
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
-    if constexpr (AB_FMT == 1) {
-      __nv_bfloat162 h = *reinterpret_cast<const __nv_bfloat162 *>(&u[i]);
-      float2 v = __bfloat1622float2(h);
-      f[2 * i] = v.x;
-      f[2 * i + 1] = v.y;
-    } else {
-      __half2 h = *reinterpret_cast<const __half2 *>(&u[i]);
-      float2 v = __half22float2(h);
-      f[2 * i] = v.x;
-      f[2 * i + 1] = v.y;
-    }
+    float2 v;
+    if constexpr (AB_FMT == 1)
+      v = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162 *>(&u[i]));
+    else
+      v = __half22float2(*reinterpret_cast<const __half2 *>(&u[i]));
+    f[2 * i] = v.x;
+    f[2 * i + 1] = v.y;
   }
 }
 
@@ -97,31 +127,41 @@ __device__ __forceinline__ uint32_t pack2(float lo, float hi) {
   }
 }
 
-// Process NU 16-byte units (8 outputs each) of this thread's row of one C chunk.
+// NU 16-byte units (8 outputs each) of this thread's row of one C chunk, starting at unit
+// u0, in place in smem.  All C_old units are read first, then computed, then written, so the
+// shared-memory accesses do not form one serial read-modify-write chain.
 template <int AB_FMT, int NU>
-__device__ __forceinline__ void epi_row(uint8_t *cb, int row, int c_swz, const uint32_t *acc, float alpha,
+__device__ __forceinline__ void epi_row(uint8_t *cb, int row, int c_swz, int u0, const uint32_t *acc, float alpha,
                                         float beta) {
+  uint32_t off[NU];
 #pragma unroll
-  for (int u = 0; u < NU; ++u) {
-    const uint32_t off = ptx::swz((uint32_t)(row * c_swz + u * 16), c_swz);
-    uint4 *p = reinterpret_cast<uint4 *>(cb + off);
-    float o[8];
-    if (beta != 0.f) {
-      float old[8];
-      unpack8<AB_FMT>(*p, old);
+  for (int u = 0; u < NU; ++u) off[u] = ptx::swz((uint32_t)(row * c_swz + (u0 + u) * 16), c_swz);
+  uint4 w[NU];
+  if (beta != 0.f) {
+#pragma unroll
+    for (int u = 0; u < NU; ++u) w[u] = *reinterpret_cast<const uint4 *>(cb + off[u]);
+#pragma unroll
+    for (int u = 0; u < NU; ++u) {
+      float old[8], o[8];
+      unpack8<AB_FMT>(w[u], old);
 #pragma unroll
       for (int e = 0; e < 8; ++e) o[e] = fmaf(alpha, __uint_as_float(acc[u * 8 + e]), beta * old[e]);
-    } else {
-#pragma unroll
-      for (int e = 0; e < 8; ++e) o[e] = alpha * __uint_as_float(acc[u * 8 + e]);
+      w[u].x = pack2<AB_FMT>(o[0], o[1]);
+      w[u].y = pack2<AB_FMT>(o[2], o[3]);
+      w[u].z = pack2<AB_FMT>(o[4], o[5]);
+      w[u].w = pack2<AB_FMT>(o[6], o[7]);
     }
-    uint4 w;
-    w.x = pack2<AB_FMT>(o[0], o[1]);
-    w.y = pack2<AB_FMT>(o[2], o[3]);
-    w.z = pack2<AB_FMT>(o[4], o[5]);
-    w.w = pack2<AB_FMT>(o[6], o[7]);
-    *p = w;
+  } else {
+#pragma unroll
+    for (int u = 0; u < NU; ++u) {
+      w[u].x = pack2<AB_FMT>(alpha * __uint_as_float(acc[u * 8 + 0]), alpha * __uint_as_float(acc[u * 8 + 1]));
+      w[u].y = pack2<AB_FMT>(alpha * __uint_as_float(acc[u * 8 + 2]), alpha * __uint_as_float(acc[u * 8 + 3]));
+      w[u].z = pack2<AB_FMT>(alpha * __uint_as_float(acc[u * 8 + 4]), alpha * __uint_as_float(acc[u * 8 + 5]));
+      w[u].w = pack2<AB_FMT>(alpha * __uint_as_float(acc[u * 8 + 6]), alpha * __uint_as_float(acc[u * 8 + 7]));
+    }
   }
+#pragma unroll
+  for (int u = 0; u < NU; ++u) *reinterpret_cast<uint4 *>(cb + off[u]) = w[u];
 }
 
 // --------------------------------------------------------------------------------- kernel
@@ -129,244 +169,375 @@ template <int AB_FMT>
 __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constant__ TcArgs p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t *stage_base = smem;
-  uint8_t *cbuf = smem + (size_t)kStages * kStageBytes;
-  Bars *bars = reinterpret_cast<Bars *>(cbuf + (size_t)kCSlots * kCSlotBytes);
+  uint8_t *pages = smem;
+  uint8_t *cbuf = smem + (size_t)kPages * kPageBytes;
+  Shared *sh = reinterpret_cast<Shared *>(cbuf + (size_t)kCSlots * kCSlotBytes);
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
 
   if (threadIdx.x == 0) {
-    for (int i = 0; i < kStages; ++i) {
-      ptx::mbar_init(&bars->full[i], 1);
-      ptx::mbar_init(&bars->empty[i], 1);
+    for (int i = 0; i < kSlots; ++i) {
+      ptx::mbar_init(&sh->full[i], 1);
+      ptx::mbar_init(&sh->empty[i], 1);
     }
     for (int i = 0; i < 2; ++i) {
-      ptx::mbar_init(&bars->tfull[i], 1);
-      ptx::mbar_init(&bars->tempty[i], 4);
+      ptx::mbar_init(&sh->tfull[i], 1);
+      ptx::mbar_init(&sh->tempty[i], kEpiWarps);
     }
     for (int i = 0; i < kCSlots; ++i) {
-      ptx::mbar_init(&bars->cfull[i], 1);
-      ptx::mbar_init(&bars->cempty[i], 1);
+      ptx::mbar_init(&sh->cfull[i], 1);
+      ptx::mbar_init(&sh->cempty[i], 4);   // one arrival per lane quarter (its storing warp)
     }
-    for (int i = 0; i < kSched; ++i) {
-      ptx::mbar_init(&bars->sfull[i], 1);
-      ptx::mbar_init(&bars->sempty[i], kSchedConsumers);
+    for (int i = 0; i < kRing; ++i) {
+      ptx::mbar_init(&sh->rfull[i], 1);
+      ptx::mbar_init(&sh->rempty[i], kRingConsumers);
     }
+    sh->prod_kb = 0u;
     ptx::fence_mbar_init();
   }
-  if (warp == 2) ptx::tmem_alloc(&bars->tmem_base, kTmemCols);
+  if (warp == 2) ptx::tmem_alloc(&sh->tmem_base, kTmemCols);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
-  const uint32_t tmem_base = bars->tmem_base;
+  const uint32_t tmem_base = sh->tmem_base;
   const uint8_t *tmaps = reinterpret_cast<const uint8_t *>(p.tmaps);
+#ifdef VB_TRACE
+  long long tr[kTraceSlots];
+  for (int i = 0; i < kTraceSlots; ++i) tr[i] = 0;
+  const long long t_start = clock64();
+#endif
 
   if (warp == 0) {
-    // ===================================================== scheduler + A/B TMA producer
+    // ================================================================ scheduler (whole warp)
+    // Tile t of this CTA goes to ring entry t % kRing with phase (t / kRing) & 1.
+    // The lookahead is bounded in k-blocks (kKbAhead) rather than tiles, so CTAs working on
+    // long-K tiles do not hoard blocks: the blocks in progress across the GPU stay a short
+    // window of consecutive GEMMs and their A/B re-reads hit in L2.
+    uint32_t t = 0, pushed_kb = 0;
+    int next = 0;
+    if (lane == 0) next = atomicAdd(p.counter, 1);
+    next = __shfl_sync(0xffffffffu, next, 0);
+    for (;;) {
+      const int b = next;
+      if (b >= p.n_blocks) break;
+      if (lane == 0) {
+        VB_TWAIT(T_SCHED_BUDGET, while ((int)(pushed_kb - sh->prod_kb) > kKbAhead) __nanosleep(128));
+        next = atomicAdd(p.counter, 1);                 // claim one block ahead
+      }
+      int lim = 0;
+      if (lane < 2) lim = p.block_ptr[b + lane];
+      const int s0 = __shfl_sync(0xffffffffu, lim, 0), s1 = __shfl_sync(0xffffffffu, lim, 1);
+      for (int base = s0; base < s1; base += 32) {
+        const int n = min(32, s1 - base);
+        int kb = 0;
+        if (lane < n) {
+          const TileDesc d = p.tiles[base + lane];
+          kb = max(d.kblocks, 1);
+          const float al = p.alpha[d.gemm], be = p.beta[d.gemm];
+          const uint32_t tt = t + lane;
+          const int e = (int)(tt % kRing);
+          VB_TWAIT(T_SCHED_REMPTY, ptx::mbar_wait(&sh->rempty[e], ((tt / kRing) & 1u) ^ 1u));
+          TileInfo &ti = sh->ring[e];
+          ti.d = d;
+          ti.alpha = al;
+          ti.beta = be;
+          ptx::mbar_arrive(&sh->rfull[e]);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) kb += __shfl_xor_sync(0xffffffffu, kb, o);
+        pushed_kb += (uint32_t)kb;
+        t += (uint32_t)n;
+      }
+      next = __shfl_sync(0xffffffffu, next, 0);
+    }
+    if (lane == 0) {                                        // end marker
+      const int e = (int)(t % kRing);
+      ptx::mbar_wait(&sh->rempty[e], ((t / kRing) & 1u) ^ 1u);
+      sh->ring[e].d.gemm = -1;
+      ptx::mbar_arrive(&sh->rfull[e]);
+    }
+  } else if (warp == 1) {
+    // ================================================================ A/B TMA producer
     if (lane == 0) {
-      int stage = 0, si = 0;
-      uint32_t phase = 0, sph = 0;
+      int re = 0, slot = 0, head = 0, oldest = 0, inflight = 0, free_pages = kPages, last_gemm = -1;
+      uint32_t rph = 0, sph = 0, ophase = 0;
+      int32_t *slot_pages = sh->slot_pages;
       for (;;) {
-        const int b = atomicAdd(p.counter, 1);
-        ptx::mbar_wait(&bars->sempty[si], sph ^ 1u);
-        bars->sched[si] = b < p.n_blocks ? b : -1;
-        ptx::mbar_arrive(&bars->sfull[si]);
-        advance(si, sph, kSched);
-        if (b >= p.n_blocks) break;
-        const int s1 = p.block_ptr[b + 1];
-        for (int s = p.block_ptr[b]; s < s1; ++s) {
-          const TileSlot ts = p.slots[s];
-          const GemmParam gp = p.gemms[ts.gemm];
-          if (gp.kblocks == 0) continue;
-          const int BY = row_BY(gp.row), BX = row_BX(gp.row);
-          const TcGeom geo = tc_geom(BY, BX);
-          const uint8_t *mapA = tmaps + (size_t)ts.gemm * 384;
-          const uint8_t *mapB = mapA + 128;
+        VB_TWAIT(T_PROD_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
+        const TileInfo ti = sh->ring[re];
+        ptx::mbar_arrive(&sh->rempty[re]);
+        advance(re, rph, kRing);
+        if (ti.d.gemm < 0) break;
+        if (ti.d.kblocks == 0) {
+          sh->prod_kb = sh->prod_kb + 1u;
+          continue;
+        }
+        const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
+        const TcGeom geo = tc_geom(BY, BX);
+        const uint8_t *mapA = tmaps + (size_t)ti.d.gemm * 384;
+        const uint8_t *mapB = mapA + 128;
+        if (ti.d.gemm != last_gemm) {
           ptx::tmap_acquire(mapA);
           ptx::tmap_acquire(mapB);
-          const uint32_t bytes = (uint32_t)(BY + BX) * kBK * 2;
-          const int y0 = ts.y * BY, x0 = ts.x * BX;
-          for (int kb = 0; kb < gp.kblocks; ++kb) {
-            ptx::mbar_wait(&bars->empty[stage], phase ^ 1u);
-            ptx::mbar_arrive_expect_tx(&bars->full[stage], bytes);
-            uint8_t *sa = stage_base + (size_t)stage * kStageBytes;
-            uint8_t *sb = sa + kABytes;
-            ptx::tma_load_2d(sa, mapA, &bars->full[stage], kb * kBK, y0);
-            for (int j = 0; j < geo.b_boxes; ++j)
-              ptx::tma_load_2d(sb + j * kBK * geo.b_swz, mapB, &bars->full[stage], x0 + j * (geo.b_swz / 2), kb * kBK);
-            advance(stage, phase, kStages);
+          last_gemm = ti.d.gemm;
+        }
+        const int a_bytes = BY * kBK * 2, b_bytes = BX * kBK * 2;
+        const int a_pages = a_bytes / kPageBytes;
+        const int need = a_pages + (b_bytes + kPageBytes - 1) / kPageBytes;
+        for (int kb = 0; kb < ti.d.kblocks; ++kb) {
+          int start = head, take = need;
+          if (start + need > kPages) {          // never wrap a k-block around the ring end
+            take += kPages - start;
+            start = 0;
           }
+          while (free_pages < take || inflight == kSlots) {
+            // reclaim the oldest k-block in flight once the MMA has consumed it
+            VB_TWAIT(T_PROD_EMPTY, ptx::mbar_wait(&sh->empty[oldest], ophase));
+            free_pages += slot_pages[oldest];
+            --inflight;
+            advance(oldest, ophase, kSlots);
+          }
+          slot_pages[slot] = take;
+          free_pages -= take;
+          ++inflight;
+          head = start + need;
+          if (head == kPages) head = 0;
+          sh->slot_page[slot] = start;
+          ptx::mbar_arrive_expect_tx(&sh->full[slot], (uint32_t)(a_bytes + b_bytes));
+          uint8_t *sa = pages + (size_t)start * kPageBytes;
+          uint8_t *sb = sa + (size_t)a_pages * kPageBytes;
+          ptx::tma_load_2d(sa, mapA, &sh->full[slot], kb * kBK, ti.d.m0);
+          for (int j = 0; j < geo.b_boxes; ++j)
+            ptx::tma_load_2d(sb + j * kBK * geo.b_swz, mapB, &sh->full[slot], ti.d.n0 + j * (geo.b_swz / 2), kb * kBK);
+          advance(slot, sph, kSlots);
+          sh->prod_kb = sh->prod_kb + 1u;
         }
       }
     }
-  } else if (warp == 1) {
-    // ===================================================== MMA issuer (single thread)
+  } else if (warp == 2) {
+    // ================================================================ MMA issuer
     if (lane == 0) {
-      int stage = 0, si = 0;
-      uint32_t phase = 0, sph = 0, t = 0;
+      int re = 0, slot = 0;
+      uint32_t rph = 0, sph = 0, t = 0;
       for (;;) {
-        ptx::mbar_wait(&bars->sfull[si], sph);
-        const int b = bars->sched[si];
-        ptx::mbar_arrive(&bars->sempty[si]);
-        advance(si, sph, kSched);
-        if (b < 0) break;
-        const int s1 = p.block_ptr[b + 1];
-        for (int s = p.block_ptr[b]; s < s1; ++s, ++t) {
-          const TileSlot ts = p.slots[s];
-          const GemmParam gp = p.gemms[ts.gemm];
-          const int BY = row_BY(gp.row), BX = row_BX(gp.row);
-          const TcGeom geo = tc_geom(BY, BX);
-          const uint32_t buf = t & 1u, aph = (t >> 1) & 1u;
-          ptx::mbar_wait(&bars->tempty[buf], aph ^ 1u);
+        VB_TWAIT(T_MMA_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
+        const TileInfo ti = sh->ring[re];
+        ptx::mbar_arrive(&sh->rempty[re]);
+        advance(re, rph, kRing);
+        if (ti.d.gemm < 0) break;
+        const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
+        const TcGeom geo = tc_geom(BY, BX);
+        const uint32_t buf = t & 1u, aph = (t >> 1) & 1u;
+        ++t;
+#ifdef VB_TRACE
+        tr[T_TILES] += 1;
+#endif
+        VB_TWAIT(T_MMA_TEMPTY, ptx::mbar_wait(&sh->tempty[buf], aph ^ 1u));
+        ptx::tc_fence_after();
+        const uint32_t d_tmem = tmem_base + buf * kAccCols;
+        const uint32_t idesc = ptx::idesc_f16((uint32_t)AB_FMT, BY, BX);
+        const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
+        const uint32_t a_bytes = (uint32_t)BY * kBK * 2;
+        for (int kb = 0; kb < ti.d.kblocks; ++kb) {
+          VB_TWAIT(T_MMA_FULL, ptx::mbar_wait(&sh->full[slot], sph));
           ptx::tc_fence_after();
-          const uint32_t d_tmem = tmem_base + buf * kAccCols;
-          const uint32_t idesc = ptx::idesc_f16((uint32_t)AB_FMT, BY, BX);
-          const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
-          for (int kb = 0; kb < gp.kblocks; ++kb) {
-            ptx::mbar_wait(&bars->full[stage], phase);
-            ptx::tc_fence_after();
-            const uint32_t sa = ptx::smem_u32(stage_base + (size_t)stage * kStageBytes);
-            const uint32_t sb = sa + kABytes;
+          const uint32_t sa = ptx::smem_u32(pages + (size_t)sh->slot_page[slot] * kPageBytes);
+          const uint32_t sb = sa + a_bytes;
 #pragma unroll
-            for (int kk = 0; kk < kBK / 16; ++kk) {
-              // A: K-major, 128-B swizzle, 8-row atoms 1024 B apart; K step of 16 = +32 B.
-              const uint64_t adesc = ptx::smem_desc(sa + kk * 32, 16, 1024, 2);
-              // B: MN-major, b_swz swizzle; 8-row (K) atoms 8*b_swz apart (SBO), MN blocks of
-              // b_swz/2 elements 64*b_swz apart (LBO); K step of 16 rows = +16*b_swz bytes.
-              const uint64_t bdesc = ptx::smem_desc(sb + kk * 16 * geo.b_swz, kBK * geo.b_swz, 8 * geo.b_swz, blayout);
-              ptx::mma_f16_ss(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
-            }
-            ptx::mma_commit(&bars->empty[stage]);   // frees the smem stage when the MMAs retire
-            advance(stage, phase, kStages);
+          for (int kk = 0; kk < kBK / 16; ++kk) {
+            // A: K-major, 128-B swizzle, 8-row atoms 1024 B apart; K step of 16 = +32 B.
+            const uint64_t adesc = ptx::smem_desc(sa + kk * 32, 16, 1024, 2);
+            // B: MN-major, b_swz swizzle; 8-row (K) atoms 8*b_swz apart (SBO), MN blocks of
+            // b_swz/2 elements 64*b_swz apart (LBO); K step of 16 rows = +16*b_swz bytes.
+            const uint64_t bdesc = ptx::smem_desc(sb + kk * 16 * geo.b_swz, kBK * geo.b_swz, 8 * geo.b_swz, blayout);
+            ptx::mma_f16_ss(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
           }
-          ptx::mma_commit(&bars->tfull[buf]);       // accumulator ready for the epilogue
+          ptx::mma_commit(&sh->empty[slot]);      // frees the k-block's pages when the MMAs retire
+          advance(slot, sph, kSlots);
         }
+        ptx::mma_commit(&sh->tfull[buf]);         // accumulator ready for the epilogue
       }
     }
   } else if (warp == 3) {
-    // ===================================================== C_old producer (beta != 0)
+    // ================================================================ C_old producer
     if (lane == 0) {
-      int cs = 0, si = 0;
-      uint32_t cph = 0, sph = 0;
+      int re = 0, cs = 0, last_gemm = -1;
+      uint32_t rph = 0, cph = 0;
       for (;;) {
-        ptx::mbar_wait(&bars->sfull[si], sph);
-        const int b = bars->sched[si];
-        ptx::mbar_arrive(&bars->sempty[si]);
-        advance(si, sph, kSched);
-        if (b < 0) break;
-        const int s1 = p.block_ptr[b + 1];
-        for (int s = p.block_ptr[b]; s < s1; ++s) {
-          const TileSlot ts = p.slots[s];
-          const GemmParam gp = p.gemms[ts.gemm];
-          const int BY = row_BY(gp.row), BX = row_BX(gp.row);
-          const TcGeom geo = tc_geom(BY, BX);
-          const float beta = p.beta[ts.gemm];
-          const uint8_t *mapC = tmaps + (size_t)ts.gemm * 384 + 256;
-          if (beta != 0.f) ptx::tmap_acquire(mapC);
-          for (int ch = 0; ch < geo.c_chunks; ++ch) {
-            ptx::mbar_wait(&bars->cempty[cs], cph ^ 1u);
-            if (beta != 0.f) {
-              ptx::mbar_arrive_expect_tx(&bars->cfull[cs], (uint32_t)(BY * geo.c_cols * 2));
-              ptx::tma_load_2d(cbuf + (size_t)cs * kCSlotBytes, mapC, &bars->cfull[cs], ts.x * BX + ch * geo.c_cols,
-                               ts.y * BY);
-            } else {
-              ptx::mbar_arrive(&bars->cfull[cs]);
-            }
-            advance(cs, cph, kCSlots);
-          }
-        }
-      }
-    }
-  } else if (warp >= 4) {
-    // ===================================================== epilogue (128 threads)
-    const int q = warp & 3;   // TMEM lane quarter this warp may access
-    const bool store_thread = (warp == 4 && lane == 0);
-    int cs = 0, si = 0;
-    uint32_t cph = 0, sph = 0, t = 0;
-    for (;;) {
-      ptx::mbar_wait(&bars->sfull[si], sph);
-      const int b = bars->sched[si];
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&bars->sempty[si]);
-      advance(si, sph, kSched);
-      if (b < 0) break;
-      const int s1 = p.block_ptr[b + 1];
-      for (int s = p.block_ptr[b]; s < s1; ++s, ++t) {
-        const TileSlot ts = p.slots[s];
-        const GemmParam gp = p.gemms[ts.gemm];
-        const int BY = row_BY(gp.row), BX = row_BX(gp.row);
+        VB_TWAIT(T_CPROD_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
+        const TileInfo ti = sh->ring[re];
+        ptx::mbar_arrive(&sh->rempty[re]);
+        advance(re, rph, kRing);
+        if (ti.d.gemm < 0) break;
+        const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
         const TcGeom geo = tc_geom(BY, BX);
-        const float alpha = p.alpha[ts.gemm], beta = p.beta[ts.gemm];
-        const uint8_t *mapC = tmaps + (size_t)ts.gemm * 384 + 256;
-        if (store_thread) ptx::tmap_acquire(mapC);
-        const uint32_t buf = t & 1u, aph = (t >> 1) & 1u;
-        ptx::mbar_wait(&bars->tfull[buf], aph);
-        ptx::tc_fence_after();
-        // M = 128: tile row 32q + lane lives in TMEM lane 32q + lane.
-        // M = 64 : tile row 16q + i lives in TMEM lane 32q + i, i < 16 (half sub-partitions).
-        const int row = BY == 128 ? q * 32 + lane : q * 16 + lane;
-        const bool row_ok = BY == 128 || lane < 16;
+        const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * 384 + 256;
+        const bool load = ti.beta != 0.f;
+        if (load && ti.d.gemm != last_gemm) {
+          ptx::tmap_acquire(mapC);
+          last_gemm = ti.d.gemm;
+        }
         for (int ch = 0; ch < geo.c_chunks; ++ch) {
-          uint32_t acc[64];
-          if (gp.kblocks > 0) {
-            const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + buf * kAccCols + ch * geo.c_cols;
-            ptx::tmem_ld_32x32b_x32(taddr, *reinterpret_cast<uint32_t(*)[32]>(&acc[0]));
-            if (geo.c_cols == 64) ptx::tmem_ld_32x32b_x32(taddr + 32, *reinterpret_cast<uint32_t(*)[32]>(&acc[32]));
-            ptx::tmem_ld_wait();
+          VB_TWAIT(T_CPROD_CEMPTY, ptx::mbar_wait(&sh->cempty[cs], cph ^ 1u));
+          if (load) {
+            // the C map's box is one epilogue warp's sub-box (BY/4 rows); skip rows >= M
+            const int rows_w = BY / 4;
+            int nsub = 0;
+            for (int w = 0; w < 4; ++w) nsub += (ti.d.m0 + w * rows_w < ti.d.M) ? 1 : 0;
+            ptx::mbar_arrive_expect_tx(&sh->cfull[cs], (uint32_t)(nsub * rows_w * geo.c_cols * 2));
+            for (int w = 0; w < nsub; ++w)
+              ptx::tma_load_2d(cbuf + (size_t)cs * kCSlotBytes + w * rows_w * geo.c_swz, mapC, &sh->cfull[cs],
+                               ti.d.n0 + ch * geo.c_cols, ti.d.m0 + w * rows_w);
           } else {
-#pragma unroll
-            for (int i = 0; i < 64; ++i) acc[i] = 0u;   // K == 0: C = beta * C
-          }
-          ptx::mbar_wait(&bars->cfull[cs], cph);
-          uint8_t *cb = cbuf + (size_t)cs * kCSlotBytes;
-          if (row_ok) {
-            if (geo.c_cols == 64)
-              epi_row<AB_FMT, 8>(cb, row, geo.c_swz, acc, alpha, beta);
-            else
-              epi_row<AB_FMT, 4>(cb, row, geo.c_swz, acc, alpha, beta);
-          }
-          const int col0 = ts.x * BX + ch * geo.c_cols;
-          if (col0 + geo.c_cols <= gp.N || (gp.N & 7) == 0) {
-            // TMA store; rows >= M and whole 16-byte granules >= N are clipped by the TMA unit.
-            ptx::fence_proxy_async_smem();
-            ptx::named_bar_sync(1, kEpiThreads);
-            if (store_thread) {
-              ptx::tma_store_2d(mapC, cb, col0, ts.y * BY);
-              ptx::bulk_commit();
-              ptx::bulk_wait_read0();
-              ptx::mbar_arrive(&bars->cempty[cs]);
-            }
-          } else {
-            // The chunk ends inside a 16-byte granule of the row (N % 8 != 0): a TMA store would
-            // write the whole granule, i.e. past N into the caller's padding.  Store this chunk
-            // from the thread's own row with exact per-element bounds instead.
-            const int grow = ts.y * BY + row;
-            if (row_ok && grow < gp.M) {
-              uint8_t *crow = static_cast<uint8_t *>(p.C[ts.gemm]) + ((size_t)grow * gp.ldc + col0) * 2;
-              const int ncol = gp.N - col0;
-              for (int u = 0; u * 8 < ncol && u * 8 < geo.c_cols; ++u) {
-                const uint4 w = *reinterpret_cast<const uint4 *>(cb + ptx::swz((uint32_t)(row * geo.c_swz + u * 16),
-                                                                                  geo.c_swz));
-                if (u * 8 + 8 <= ncol) {
-                  *reinterpret_cast<uint4 *>(crow + u * 16) = w;
-                } else {
-                  const uint16_t *h = reinterpret_cast<const uint16_t *>(&w);
-                  for (int e = 0; e < ncol - u * 8; ++e) reinterpret_cast<uint16_t *>(crow + u * 16)[e] = h[e];
-                }
-              }
-            }
-            ptx::named_bar_sync(1, kEpiThreads);
-            if (store_thread) ptx::mbar_arrive(&bars->cempty[cs]);
+            ptx::mbar_arrive(&sh->cfull[cs]);
           }
           advance(cs, cph, kCSlots);
         }
-        ptx::tc_fence_before();
-        __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&bars->tempty[buf]);
       }
     }
-    if (store_thread) ptx::bulk_wait0();
+  } else {
+    // ================================================================ epilogue (8 warps)
+    // Warps 4+q and 8+q share TMEM lane quarter q (tile rows r0 .. r0+BY/4-1) and split each
+    // chunk's columns in halves.  The pair meets on a 64-thread named barrier per chunk, then
+    // warp 4+q TMA-stores the quarter's sub-box itself: no barrier spans all epilogue warps,
+    // and TMEM loads of the next chunk are issued before the current one is processed.
+    const int q = warp & 3;
+    const int half = (warp - 4) >> 2;
+    const bool storer = half == 0;
+    int re = 0, cs = 0, pending = -1, last_gemm = -1;
+    uint32_t rph = 0, cph = 0, t = 0;
+    for (;;) {
+      VB_TWAIT(T_EPI_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
+      const TileInfo ti = sh->ring[re];
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&sh->rempty[re]);
+      advance(re, rph, kRing);
+      if (ti.d.gemm < 0) break;
+      const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
+      const TcGeom geo = tc_geom(BY, BX);
+      const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * 384 + 256;
+      if (storer && lane == 0 && ti.d.gemm != last_gemm) {
+        ptx::tmap_acquire(mapC);
+        last_gemm = ti.d.gemm;
+      }
+      const uint32_t buf = t & 1u, aph = (t >> 1) & 1u;
+      ++t;
+      // M = 128: tile row 32q + i lives in TMEM lane 32q + i.
+      // M = 64 : tile row 16q + i lives in TMEM lane 32q + i, i < 16 (half sub-partitions).
+      const int rows_w = BY / 4;
+      const int r0 = q * rows_w;
+      const int row = r0 + lane;
+      const bool row_ok = lane < rows_w;
+      const bool live = ti.d.m0 + r0 < ti.d.M;          // any row of this quarter inside the GEMM
+      const bool has_acc = ti.d.kblocks > 0;
+      const int hcols = geo.c_cols / 2;                  // this warp's columns of a chunk
+      const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + buf * kAccCols + half * hcols;
+      VB_TWAIT(T_EPI_TFULL, ptx::mbar_wait(&sh->tfull[buf], aph));
+      ptx::tc_fence_after();
+
+      auto tload = [&](int ch, uint32_t *acc) {
+        const uint32_t ta = tbase + ch * geo.c_cols;
+        if (hcols == 32)
+          ptx::tmem_ld_32x32b_x32(ta, *reinterpret_cast<uint32_t(*)[32]>(acc));
+        else
+          ptx::tmem_ld_32x32b_x16(ta, acc);
+      };
+      auto release_acc = [&]() {                       // accumulator drained: hand it back early
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&sh->tempty[buf]);
+      };
+      auto process = [&](int ch, const uint32_t *acc) {
+        const int col0 = ti.d.n0 + ch * geo.c_cols;
+        const bool direct = (ti.d.flags & 1) && (col0 + geo.c_cols > ti.d.N);
+        if (storer && lane == 0 && direct && pending >= 0) {   // keep at most one store pending
+          ptx::bulk_wait_read0();
+          ptx::mbar_arrive(&sh->cempty[pending]);
+          pending = -1;
+        }
+        VB_TWAIT(T_EPI_CFULL, ptx::mbar_wait(&sh->cfull[cs], cph));
+        uint8_t *cb = cbuf + (size_t)cs * kCSlotBytes;
+        {
+          VB_T0();
+          if (row_ok && live) {
+            if (hcols == 32)
+              epi_row<AB_FMT, 4>(cb, row, geo.c_swz, half * 4, acc, ti.alpha, ti.beta);
+            else
+              epi_row<AB_FMT, 2>(cb, row, geo.c_swz, half * 2, acc, ti.alpha, ti.beta);
+          }
+          VB_TADD(T_EPI_MATH);
+        }
+        if (!direct) {
+          // TMA store of the quarter's sub-box; rows >= M and whole 16-byte granules >= N are
+          // clipped by the TMA unit.
+          ptx::fence_proxy_async_smem();
+          ptx::named_bar_sync(1 + q, 64);
+          if (storer && lane == 0) {
+            if (live) {
+              ptx::tma_store_2d(mapC, cb + r0 * geo.c_swz, col0, ti.d.m0 + r0);
+              ptx::bulk_commit();
+            }
+            if (pending >= 0) {
+              VB_TWAIT(T_EPI_STORE, ptx::bulk_wait_read1());   // the previous store has read its slot
+              ptx::mbar_arrive(&sh->cempty[pending]);
+            }
+            pending = cs;
+          }
+        } else {
+          // The chunk ends inside a 16-byte granule of the row (N % 8 != 0): a TMA store would
+          // write the whole granule, past N into the caller's padding.  Store this warp's
+          // columns from the thread's own row with exact per-element bounds instead.
+          const int grow = ti.d.m0 + row;
+          if (row_ok && grow < ti.d.M) {
+            const int c_lo = half * hcols;
+            uint8_t *crow = static_cast<uint8_t *>(p.C[ti.d.gemm]) + ((size_t)grow * ti.d.ldc + col0) * 2;
+            const int ncol = min(ti.d.N - col0, c_lo + hcols);
+            for (int c = c_lo; c < ncol; c += 8) {
+              const uint4 w =
+                  *reinterpret_cast<const uint4 *>(cb + ptx::swz((uint32_t)(row * geo.c_swz + c * 2), geo.c_swz));
+              if (c + 8 <= ncol) {
+                *reinterpret_cast<uint4 *>(crow + c * 2) = w;
+              } else {
+                const uint16_t *h = reinterpret_cast<const uint16_t *>(&w);
+                for (int e = 0; e < ncol - c; ++e) reinterpret_cast<uint16_t *>(crow + c * 2)[e] = h[e];
+              }
+            }
+          }
+          ptx::named_bar_sync(1 + q, 64);
+          if (storer && lane == 0) ptx::mbar_arrive(&sh->cempty[cs]);
+        }
+        advance(cs, cph, kCSlots);
+      };
+
+      uint32_t a0[32], a1[32];
+      const int nch = geo.c_chunks;
+      if (has_acc) {
+        tload(0, a0);
+      } else {
+#pragma unroll
+        for (int i = 0; i < 32; ++i) a0[i] = a1[i] = 0u;   // K == 0: C = beta * C
+      }
+      for (int ch = 0; ch < nch; ch += 2) {
+        if (has_acc) VB_TWAIT(T_EPI_TMEM, ptx::tmem_ld_wait());
+        if (has_acc && ch + 1 < nch) tload(ch + 1, a1);
+        if (ch + 1 >= nch) release_acc();
+        process(ch, a0);
+        if (ch + 1 < nch) {
+          if (has_acc) VB_TWAIT(T_EPI_TMEM, ptx::tmem_ld_wait());
+          if (has_acc && ch + 2 < nch) tload(ch + 2, a0);
+          if (ch + 2 >= nch) release_acc();
+          process(ch + 1, a1);
+        }
+      }
+    }
+    if (storer && lane == 0) ptx::bulk_wait0();
   }
+#ifdef VB_TRACE
+  tr[T_TOTAL] = clock64() - t_start;
+  if (lane == 0 && p.trace)
+    for (int i = 0; i < kTraceSlots; ++i)
+      if (tr[i]) atomicAdd(reinterpret_cast<unsigned long long *>(p.trace) + i, (unsigned long long)tr[i]);
+#endif
   __syncwarp();
   ptx::tc_fence_before();
   __syncthreads();
@@ -384,8 +555,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   }
 }
 
-// Exec-time prep: patch the global address of every per-GEMM tensor map (A, B, C) with the
-// caller's pointers (tensormap.replace), and reset the dynamic work-list counter.
+// Bind-time prep: patch the global address of every per-GEMM tensor map (A, B, C) with the
+// caller's pointers (tensormap.replace), and reset the dynamic work-list counters.
 __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
                            const GemmParam *gemms, int batch, int32_t *counter) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;

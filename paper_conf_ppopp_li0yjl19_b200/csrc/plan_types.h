@@ -36,16 +36,30 @@ struct F32Args {
   const float *beta;
 };
 
+// Per tile slot, precomputed by the planner for the tensor-core kernel: the five arrays of
+// Fig. 6 joined with the per-GEMM sizes, so the kernel reads one 32-byte record per tile.
+struct alignas(16) TileDesc {
+  int32_t gemm;
+  int32_t m0;        // element row of the tile origin    (Y_Coord * BY)
+  int32_t n0;        // element column of the tile origin (X_Coord * BX)
+  int32_t kblocks;   // ceil(K / 64)
+  int32_t M, N;      // GEMM extents
+  int32_t ldc;       // elements
+  uint16_t geo;      // (BY / 16) | (BX / 16) << 8
+  uint16_t flags;    // bit 0: the tile's last C chunk ends inside a 16-byte granule (N % 8 != 0)
+};
+static_assert(sizeof(TileDesc) == 32, "TileDesc must stay 32 bytes");
+
 struct TcArgs {
   const int32_t *block_ptr;
-  const TileSlot *slots;
-  const GemmParam *gemms;
+  const TileDesc *tiles;    // [n_slots]
   const void *tmaps;        // CUtensorMap[batch][3] = {A, B, C}, 128-byte aligned
   void *const *C;           // C pointers (direct stores of row tails that TMA cannot clip)
   const float *alpha;
   const float *beta;
-  int32_t *counter;         // dynamic work-list counter (reset by the prep kernel)
+  int32_t *counter;         // [0] dynamic work-list counter, [1] finished CTAs
   int32_t n_blocks;
+  long long *trace;         // VB_TRACE builds only: per-role wait cycles (else nullptr)
 };
 
 // Tensor-core strategy geometry derived from a table row (BY, BX): TMA boxes and swizzles.

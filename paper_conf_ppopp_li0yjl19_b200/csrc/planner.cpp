@@ -34,13 +34,15 @@ int64_t tlp_eq1(const int32_t *M, const int32_t *N, int batch, const std::vector
 TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const TableDef &t,
                         int64_t threshold) {
   const std::vector<int> order = priority_order(t);
-  // Step 1 (P249): per-GEMM queue of strategies with BY <= M and BX <= N (C-1); if none
+  // Step 1 (P249): per-GEMM queue of strategies with BY <= M and BX <= N (C-1, with the
+  // table's MMA floor C-1b); if none
   // fits, the smallest strategy alone (C-4).  A queue is a [head, end) window of `order`
   // restricted to fitting rows, so pop = advance head, top = read head.
   std::vector<std::vector<int>> q(batch);
   for (int i = 0; i < batch; ++i) {
+    const int mf = std::max<int>(M[i], t.min_BY), nf = std::max<int>(N[i], t.min_BX);   // C-1b floor
     for (int r : order)
-      if (t.rows[r].BY <= M[i] && t.rows[r].BX <= N[i]) q[i].push_back(r);
+      if (t.rows[r].BY <= mf && t.rows[r].BX <= nf) q[i].push_back(r);
     if (q[i].empty()) q[i].push_back(order[0]);
   }
   std::vector<size_t> head(batch, 0);
@@ -49,6 +51,9 @@ TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const Tab
   out.row.assign(batch, 0);
   for (;;) {
     // Step 2: pop one strategy per GEMM, or top when a single one is left (exception 1, C-2).
+    bool single_before = true;
+    for (int i = 0; i < batch; ++i)
+      if (q[i].size() - head[i] > 1) single_before = false;
     bool all_single = true;
     for (int i = 0; i < batch; ++i) {
       out.row[i] = q[i][head[i]];
@@ -62,10 +67,14 @@ TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const Tab
     // Step 3: compare with the threshold (strict, C-6).
     if (tlp <= threshold) return out;
     // Exception 2 (C-7): about to repeat step 2 while every queue holds one strategy:
-    // switch to the next thread version; with no further version, stop.
+    // switch to the next thread version and repeat.  With no further version, repeat once
+    // more if this round popped (the largest strategies get evaluated); if this round already
+    // took every queue's top, nothing larger exists and the solution stands.
     if (all_single) {
-      if (vi + 1 >= t.n_versions) return out;
-      ++vi;
+      if (vi + 1 < t.n_versions)
+        ++vi;
+      else if (single_before)
+        return out;
     }
   }
 }

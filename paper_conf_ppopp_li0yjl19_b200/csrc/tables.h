@@ -12,7 +12,7 @@ struct StrategyRow {
   int BK;   // K step of one main-loop iteration
 };
 
-constexpr int kMaxRows = 6;
+constexpr int kMaxRows = 8;
 constexpr int kMaxVersions = 2;
 
 struct TableDef {
@@ -24,6 +24,12 @@ struct TableDef {
   int versions[kMaxVersions];   // thread counts T, preferred (more TLP) first — P247
   int64_t tlp_threshold;        // P253 / P290 (platform constant)
   int theta;                    // P259 / P290 (platform constant)
+  // Availability floor (reading C-1b): a strategy is available for a GEMM when
+  // BY <= max(M, min_BY) and BX <= max(N, min_BX).  0 for the paper's tables (P249 exactly);
+  // for tcgen05 the MMA cannot be shorter than 64 rows, so min_BY = 64 (and min_BX = 32,
+  // the narrowest strategy): a 20-row GEMM occupies a 64-row MMA whichever tile it gets.
+  int min_BY;
+  int min_BX;
 };
 
 // PAPER.md Table 2 (P204-214): small 16x16, medium 32x32, large 64x64, tall 128x64,
@@ -33,18 +39,20 @@ struct TableDef {
    {"tall", 128, 64, 8}, {"wide", 64, 128, 8}, {"huge", 128, 128, 8}}
 
 // V100 profile: the paper's constants (P255, P290).
-constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 128}, 65536, 256};
+constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 128}, 65536, 256, 0, 0};
 
 // B200 FFMA profile (fp32): Table 2 shapes/sub-tiles (an FFMA design that still holds on
 // sm_100a), threshold re-set for 148 SMs (reading C-22, calibration is NEXT-1).
-constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 2, {256, 128}, 131072, 256};
+constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 2, {256, 128}, 131072, 256, 0, 0};
 
-// B200 tcgen05 profile (bf16/fp16): tcgen05.mma M in {64,128}; BK = 64 = one 128-byte
-// swizzled row of bf16; one kernel version with 256 threads (8 warps).
-constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 6,
-                                   {{"s", 64, 32, 64}, {"m", 64, 64, 64}, {"t", 128, 64, 64},
-                                    {"w", 64, 128, 64}, {"l", 128, 128, 64}, {"h", 128, 256, 64}},
-                                   1, {256, 0}, 4 * 148 * 256, 512};
+// B200 tcgen05 profile (bf16/fp16): C tiles for tcgen05.mma with M in {64,128}; BK = 64 =
+// one 128-byte swizzled row of bf16; one kernel version with 256 threads (8 warps).  Besides
+// the paper's square/tall/wide family it has the skinny shapes 128x32 and 64x256 that
+// variable-size batches need once short GEMMs may take the 64-row MMA (min_BY = 64).
+constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 8,
+                                   {{"s", 64, 32, 64}, {"n", 128, 32, 64}, {"m", 64, 64, 64}, {"t", 128, 64, 64},
+                                    {"w", 64, 128, 64}, {"l", 128, 128, 64}, {"x", 64, 256, 64}, {"h", 128, 256, 64}},
+                                   1, {256, 0}, 4 * 148 * 256, 512, 64, 32};
 
 #undef VB_TABLE2_ROWS
 

@@ -120,13 +120,13 @@ def _forced_rows_plan(db, rows, table, table_id):
 def test_every_strategy_row_forced(dtype):
     # every row of the table on ragged shapes, including shapes smaller than the tile
     rng = np.random.default_rng(4)
-    n = 36
+    n = 48
     M = rng.integers(1, 400, n); N = rng.integers(1, 400, n); K = rng.integers(0, 600, n)
     db = DeviceBatch(M, N, K, dtype)
     db.C.fill_(float("nan"))
     db.fill(SEED)
     table, tid = (pr.B200_TC, 3) if dtype != "f32" else (pr.B200_F32, 2)
-    rows = [g % 6 for g in range(n)]
+    rows = [g % len(table.rows) for g in range(n)]
     db.run(_forced_rows_plan(db, rows, table, tid))
     torch.cuda.synchronize()
     check_batch(db, range(n), SEED, "random")
