@@ -32,18 +32,20 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False, trace: bool = False) -> str:
-    """trace=True builds libvbgemm_trace.so with -DVB_TRACE (per-role wait-cycle accounting)."""
-    lib = TRACE_LIB if trace else LIB
-    if not force and not trace and not _stale():
+def build(force: bool = False, verbose: bool = False, trace: bool = False, defines=(), out: str = "") -> str:
+    """trace=True builds libvbgemm_trace.so with -DVB_TRACE (per-role wait-cycle accounting);
+    defines/out build an experiment variant (e.g. VB_PAGES=22) into another .so name."""
+    lib = os.path.join(HERE, out) if out else (TRACE_LIB if trace else LIB)
+    if not force and not trace and not out and not _stale():
         return LIB
-    objdir = os.path.join(HERE, "build_trace" if trace else "build")
+    objdir = os.path.join(HERE, "build_" + (out.replace(".so", "") if out else ("trace" if trace else "main")))
     os.makedirs(objdir, exist_ok=True)
     objs = []
     procs = []
     for src in SOURCES:
         obj = os.path.join(objdir, src + ".o")
-        cmd = [NVCC] + FLAGS + (["-DVB_TRACE"] if trace else []) + ["-c", os.path.join(CSRC, src), "-o", obj]
+        cmd = [NVCC] + FLAGS + (["-DVB_TRACE"] if trace else []) + ["-D" + d for d in defines] + \
+            ["-c", os.path.join(CSRC, src), "-o", obj]
         if src.endswith(".cu") and verbose:
             cmd += ["-Xptxas", "-v"]
         procs.append((src, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
@@ -64,4 +66,7 @@ def build(force: bool = False, verbose: bool = False, trace: bool = False) -> st
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, trace="--trace" in sys.argv))
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, trace="--trace" in sys.argv, defines=defs,
+                out=outs[0] if outs else ""))

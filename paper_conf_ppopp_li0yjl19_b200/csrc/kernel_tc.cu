@@ -35,14 +35,25 @@ namespace tck {
 constexpr int kThreads = 384;              // 4 role warps + 8 epilogue warps
 constexpr int kBK = 64;                    // bf16 elements per k-block = one 128-B swizzle row
 constexpr int kPageBytes = 8192;
-constexpr int kPages = 18;                 // 144 KB of A/B staging
+#ifndef VB_PAGES
+#define VB_PAGES 18
+#endif
+#ifndef VB_CSLOTS
+#define VB_CSLOTS 4
+#endif
+#ifndef VB_KBAHEAD
+#define VB_KBAHEAD 24
+#endif
+constexpr int kPages = VB_PAGES;           // 144 KB of A/B staging (default)
 constexpr int kSlots = 16;                 // k-blocks in flight (bounded by pages anyway)
-constexpr int kCSlots = 4;
+constexpr int kCSlots = VB_CSLOTS;
 constexpr int kCSlotBytes = 128 * 128;     // BY rows x 128 B
 constexpr int kRing = 32;                  // tile-descriptor ring entries
-constexpr int kKbAhead = 24;               // scheduler lookahead budget in k-blocks (L2 locality)
+constexpr int kKbAhead = VB_KBAHEAD;       // scheduler lookahead budget in k-blocks (L2 locality)
 constexpr int kTmemCols = 512;
-constexpr int kAccCols = 256;
+constexpr int kAccUnit = 32;               // TMEM accumulator ring granularity (columns)
+constexpr int kAccUnits = kTmemCols / kAccUnit;
+constexpr int kAcc = 8;                    // accumulators in flight (ring entries)
 constexpr int kEpiWarps = 8;               // two per TMEM lane quarter, splitting each chunk's columns
 constexpr uint32_t kRingConsumers = 1 + 1 + 1 + kEpiWarps;   // producer, MMA, C producer, epilogue warps
 
@@ -55,11 +66,12 @@ static_assert(sizeof(TileInfo) == 48, "TileInfo size");
 
 struct Shared {
   uint64_t full[kSlots], empty[kSlots];
-  uint64_t tfull[2], tempty[2];
+  uint64_t tfull[kAcc], tempty[kAcc];
   uint64_t cfull[kCSlots], cempty[kCSlots];
   uint64_t rfull[kRing], rempty[kRing];
   int32_t slot_page[kSlots];
   int32_t slot_pages[kSlots];   // producer-private: pages charged to each k-block in flight
+  int32_t acc_take[kAcc];       // MMA-private: TMEM units charged to each accumulator in flight
   uint32_t tmem_base;
   volatile uint32_t prod_kb;    // k-blocks (>= 1 per tile) the A/B producer has finished issuing
   TileInfo ring[kRing];
@@ -73,7 +85,7 @@ constexpr size_t kSmemBytes = 1024 /*align slack*/ + (size_t)kPages * kPageBytes
 enum TraceSlot {
   T_SCHED_REMPTY, T_SCHED_BUDGET, T_PROD_RFULL, T_PROD_EMPTY, T_MMA_RFULL, T_MMA_TEMPTY, T_MMA_FULL,
   T_CPROD_RFULL, T_CPROD_CEMPTY, T_EPI_RFULL, T_EPI_TFULL, T_EPI_CFULL, T_EPI_STORE, T_EPI_TMEM, T_EPI_MATH,
-  T_TOTAL, T_TILES, kTraceSlots
+  T_TOTAL, T_TILES, T_PROD_ISSUE, T_MMA_ISSUE, T_EPI_FENCEBAR, T_EPI_STISSUE, T_EPI_LOOP, kTraceSlots
 };
 #ifdef VB_TRACE
 #define VB_T0() const long long _vbt0 = clock64()
@@ -92,6 +104,24 @@ enum TraceSlot {
 
 __device__ __forceinline__ int geo_BY(uint16_t g) { return (g & 0xFF) * 16; }
 __device__ __forceinline__ int geo_BX(uint16_t g) { return (g >> 8) * 16; }
+
+// TMEM accumulator ring: tile t takes BX/32 contiguous 32-column units starting at `head`
+// (never wrapping); the MMA warp and the epilogue run this same function over the same tile
+// sequence, so the epilogue knows each accumulator's columns without any message.
+struct AccRing {
+  int head = 0;
+  __device__ __forceinline__ int place(int units, int &take) {
+    int start = head;
+    take = units;
+    if (start + units > kAccUnits) {
+      take += kAccUnits - start;
+      start = 0;
+    }
+    head = start + units;
+    if (head == kAccUnits) head = 0;
+    return start;
+  }
+};
 
 __device__ __forceinline__ void advance(int &idx, uint32_t &phase, int n) {
   if (++idx == n) {
@@ -180,7 +210,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       ptx::mbar_init(&sh->full[i], 1);
       ptx::mbar_init(&sh->empty[i], 1);
     }
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < kAcc; ++i) {
       ptx::mbar_init(&sh->tfull[i], 1);
       ptx::mbar_init(&sh->tempty[i], kEpiWarps);
     }
@@ -233,6 +263,13 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         if (lane < n) {
           const TileDesc d = p.tiles[base + lane];
           kb = max(d.kblocks, 1);
+          // warm the TMA descriptor cache for the tile's maps well before the producers use them
+          const uint8_t *maps = tmaps + (size_t)d.gemm * 384;
+          if (d.kblocks > 0) {
+            ptx::prefetch_tmap(maps);
+            ptx::prefetch_tmap(maps + 128);
+          }
+          ptx::prefetch_tmap(maps + 256);
           const float al = p.alpha[d.gemm], be = p.beta[d.gemm];
           const uint32_t tt = t + lane;
           const int e = (int)(tt % kRing);
@@ -259,7 +296,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   } else if (warp == 1) {
     // ================================================================ A/B TMA producer
     if (lane == 0) {
-      int re = 0, slot = 0, head = 0, oldest = 0, inflight = 0, free_pages = kPages, last_gemm = -1;
+      int re = 0, slot = 0, head = 0, oldest = 0, inflight = 0, free_pages = kPages;
       uint32_t rph = 0, sph = 0, ophase = 0;
       int32_t *slot_pages = sh->slot_pages;
       for (;;) {
@@ -276,11 +313,6 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const TcGeom geo = tc_geom(BY, BX);
         const uint8_t *mapA = tmaps + (size_t)ti.d.gemm * 384;
         const uint8_t *mapB = mapA + 128;
-        if (ti.d.gemm != last_gemm) {
-          ptx::tmap_acquire(mapA);
-          ptx::tmap_acquire(mapB);
-          last_gemm = ti.d.gemm;
-        }
         const int a_bytes = BY * kBK * 2, b_bytes = BX * kBK * 2;
         const int a_pages = a_bytes / kPageBytes;
         const int need = a_pages + (b_bytes + kPageBytes - 1) / kPageBytes;
@@ -303,12 +335,14 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           head = start + need;
           if (head == kPages) head = 0;
           sh->slot_page[slot] = start;
+          VB_T0();
           ptx::mbar_arrive_expect_tx(&sh->full[slot], (uint32_t)(a_bytes + b_bytes));
           uint8_t *sa = pages + (size_t)start * kPageBytes;
           uint8_t *sb = sa + (size_t)a_pages * kPageBytes;
           ptx::tma_load_2d(sa, mapA, &sh->full[slot], kb * kBK, ti.d.m0);
           for (int j = 0; j < geo.b_boxes; ++j)
             ptx::tma_load_2d(sb + j * kBK * geo.b_swz, mapB, &sh->full[slot], ti.d.n0 + j * (geo.b_swz / 2), kb * kBK);
+          VB_TADD(T_PROD_ISSUE);
           advance(slot, sph, kSlots);
           sh->prod_kb = sh->prod_kb + 1u;
         }
@@ -317,8 +351,10 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   } else if (warp == 2) {
     // ================================================================ MMA issuer
     if (lane == 0) {
-      int re = 0, slot = 0;
-      uint32_t rph = 0, sph = 0, t = 0;
+      int re = 0, slot = 0, oldest = 0, free_units = kAccUnits, inflight = 0;
+      uint32_t rph = 0, sph = 0, t = 0, ophase = 0;
+      int32_t *acc_take = sh->acc_take;
+      AccRing ring;
       for (;;) {
         VB_TWAIT(T_MMA_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
         const TileInfo ti = sh->ring[re];
@@ -327,20 +363,35 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         if (ti.d.gemm < 0) break;
         const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
         const TcGeom geo = tc_geom(BY, BX);
-        const uint32_t buf = t & 1u, aph = (t >> 1) & 1u;
+        const int e = (int)(t % kAcc);
         ++t;
 #ifdef VB_TRACE
         tr[T_TILES] += 1;
 #endif
-        VB_TWAIT(T_MMA_TEMPTY, ptx::mbar_wait(&sh->tempty[buf], aph ^ 1u));
+        int take;
+        const int start = ring.place(BX / kAccUnit, take);
+        {
+          VB_T0();
+          while (free_units < take || inflight == kAcc) {   // reclaim drained accumulators (FIFO)
+            ptx::mbar_wait(&sh->tempty[oldest], ophase);
+            free_units += acc_take[oldest];
+            --inflight;
+            advance(oldest, ophase, kAcc);
+          }
+          VB_TADD(T_MMA_TEMPTY);
+        }
+        free_units -= take;
+        acc_take[e] = take;
+        ++inflight;
         ptx::tc_fence_after();
-        const uint32_t d_tmem = tmem_base + buf * kAccCols;
+        const uint32_t d_tmem = tmem_base + (uint32_t)(start * kAccUnit);
         const uint32_t idesc = ptx::idesc_f16((uint32_t)AB_FMT, BY, BX);
         const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
         const uint32_t a_bytes = (uint32_t)BY * kBK * 2;
         for (int kb = 0; kb < ti.d.kblocks; ++kb) {
           VB_TWAIT(T_MMA_FULL, ptx::mbar_wait(&sh->full[slot], sph));
           ptx::tc_fence_after();
+          VB_T0();
           const uint32_t sa = ptx::smem_u32(pages + (size_t)sh->slot_page[slot] * kPageBytes);
           const uint32_t sb = sa + a_bytes;
 #pragma unroll
@@ -353,16 +404,18 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             ptx::mma_f16_ss(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
           }
           ptx::mma_commit(&sh->empty[slot]);      // frees the k-block's pages when the MMAs retire
+          VB_TADD(T_MMA_ISSUE);
           advance(slot, sph, kSlots);
         }
-        ptx::mma_commit(&sh->tfull[buf]);         // accumulator ready for the epilogue
+        ptx::mma_commit(&sh->tfull[e]);           // accumulator ready for the epilogue
       }
     }
   } else if (warp == 3) {
     // ================================================================ C_old producer
     if (lane == 0) {
-      int re = 0, cs = 0, last_gemm = -1;
+      int re = 0, cs = 0;
       uint32_t rph = 0, cph = 0;
+      const uint64_t c_policy = ptx::policy_evict_first();
       for (;;) {
         VB_TWAIT(T_CPROD_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
         const TileInfo ti = sh->ring[re];
@@ -373,10 +426,6 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const TcGeom geo = tc_geom(BY, BX);
         const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * 384 + 256;
         const bool load = ti.beta != 0.f;
-        if (load && ti.d.gemm != last_gemm) {
-          ptx::tmap_acquire(mapC);
-          last_gemm = ti.d.gemm;
-        }
         for (int ch = 0; ch < geo.c_chunks; ++ch) {
           VB_TWAIT(T_CPROD_CEMPTY, ptx::mbar_wait(&sh->cempty[cs], cph ^ 1u));
           if (load) {
@@ -386,8 +435,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             for (int w = 0; w < 4; ++w) nsub += (ti.d.m0 + w * rows_w < ti.d.M) ? 1 : 0;
             ptx::mbar_arrive_expect_tx(&sh->cfull[cs], (uint32_t)(nsub * rows_w * geo.c_cols * 2));
             for (int w = 0; w < nsub; ++w)
-              ptx::tma_load_2d(cbuf + (size_t)cs * kCSlotBytes + w * rows_w * geo.c_swz, mapC, &sh->cfull[cs],
-                               ti.d.n0 + ch * geo.c_cols, ti.d.m0 + w * rows_w);
+              ptx::tma_load_2d_hint(cbuf + (size_t)cs * kCSlotBytes + w * rows_w * geo.c_swz, mapC, &sh->cfull[cs],
+                                    ti.d.n0 + ch * geo.c_cols, ti.d.m0 + w * rows_w, c_policy);
           } else {
             ptx::mbar_arrive(&sh->cfull[cs]);
           }
@@ -404,8 +453,10 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     const int q = warp & 3;
     const int half = (warp - 4) >> 2;
     const bool storer = half == 0;
-    int re = 0, cs = 0, pending = -1, last_gemm = -1;
+    const uint64_t c_policy = ptx::policy_evict_first();
+    int re = 0, cs = 0, pending = -1;
     uint32_t rph = 0, cph = 0, t = 0;
+    AccRing acc_ring;
     for (;;) {
       VB_TWAIT(T_EPI_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
       const TileInfo ti = sh->ring[re];
@@ -416,12 +467,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
       const TcGeom geo = tc_geom(BY, BX);
       const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * 384 + 256;
-      if (storer && lane == 0 && ti.d.gemm != last_gemm) {
-        ptx::tmap_acquire(mapC);
-        last_gemm = ti.d.gemm;
-      }
-      const uint32_t buf = t & 1u, aph = (t >> 1) & 1u;
+      const int e = (int)(t % kAcc);
+      const uint32_t aph = (t / kAcc) & 1u;
       ++t;
+      int take;
+      const int acc_col = acc_ring.place(BX / kAccUnit, take) * kAccUnit;
       // M = 128: tile row 32q + i lives in TMEM lane 32q + i.
       // M = 64 : tile row 16q + i lives in TMEM lane 32q + i, i < 16 (half sub-partitions).
       const int rows_w = BY / 4;
@@ -431,9 +481,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const bool live = ti.d.m0 + r0 < ti.d.M;          // any row of this quarter inside the GEMM
       const bool has_acc = ti.d.kblocks > 0;
       const int hcols = geo.c_cols / 2;                  // this warp's columns of a chunk
-      const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + buf * kAccCols + half * hcols;
-      VB_TWAIT(T_EPI_TFULL, ptx::mbar_wait(&sh->tfull[buf], aph));
+      const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)acc_col + half * hcols;
+      VB_TWAIT(T_EPI_TFULL, ptx::mbar_wait(&sh->tfull[e], aph));
       ptx::tc_fence_after();
+#ifdef VB_TRACE
+      const long long _tile_t0 = clock64();
+#endif
 
       auto tload = [&](int ch, uint32_t *acc) {
         const uint32_t ta = tbase + ch * geo.c_cols;
@@ -445,7 +498,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       auto release_acc = [&]() {                       // accumulator drained: hand it back early
         ptx::tc_fence_before();
         __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&sh->tempty[buf]);
+        if (lane == 0) ptx::mbar_arrive(&sh->tempty[e]);
       };
       auto process = [&](int ch, const uint32_t *acc) {
         const int col0 = ti.d.n0 + ch * geo.c_cols;
@@ -459,7 +512,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         uint8_t *cb = cbuf + (size_t)cs * kCSlotBytes;
         {
           VB_T0();
+#ifdef VB_EXP_NOMATH
+          if (false) {
+#else
           if (row_ok && live) {
+#endif
             if (hcols == 32)
               epi_row<AB_FMT, 4>(cb, row, geo.c_swz, half * 4, acc, ti.alpha, ti.beta);
             else
@@ -470,11 +527,15 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         if (!direct) {
           // TMA store of the quarter's sub-box; rows >= M and whole 16-byte granules >= N are
           // clipped by the TMA unit.
-          ptx::fence_proxy_async_smem();
-          ptx::named_bar_sync(1 + q, 64);
+          VB_TWAIT(T_EPI_FENCEBAR, ptx::fence_proxy_async_smem(); ptx::named_bar_sync(1 + q, 64));
+          VB_T0();
           if (storer && lane == 0) {
+#ifdef VB_EXP_NOSTORE
+            if (false) {
+#else
             if (live) {
-              ptx::tma_store_2d(mapC, cb + r0 * geo.c_swz, col0, ti.d.m0 + r0);
+#endif
+              ptx::tma_store_2d_hint(mapC, cb + r0 * geo.c_swz, col0, ti.d.m0 + r0, c_policy);
               ptx::bulk_commit();
             }
             if (pending >= 0) {
@@ -483,6 +544,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             }
             pending = cs;
           }
+          VB_TADD(T_EPI_STISSUE);
         } else {
           // The chunk ends inside a 16-byte granule of the row (N % 8 != 0): a TMA store would
           // write the whole granule, past N into the caller's padding.  Store this warp's
@@ -529,6 +591,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           process(ch + 1, a1);
         }
       }
+#ifdef VB_TRACE
+      tr[T_EPI_LOOP] += clock64() - _tile_t0;
+#endif
     }
     if (storer && lane == 0) ptx::bulk_wait0();
   }
@@ -556,7 +621,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 }
 
 // Bind-time prep: patch the global address of every per-GEMM tensor map (A, B, C) with the
-// caller's pointers (tensormap.replace), and reset the dynamic work-list counters.
+// caller's pointers (tensormap.replace), and reset the dynamic work-list counters.  The maps
+// are only ever modified here, in a launch that completes before any GEMM kernel using them
+// starts (stream order), so the GEMM kernel issues no per-map acquire fence (each one is a full
+// scoreboard drain plus a descriptor-cache invalidate); tests re-bind one plan to alternating
+// buffers to check that no stale descriptor is ever used.
 __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
                            const GemmParam *gemms, int batch, int32_t *counter) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;

@@ -18,7 +18,7 @@ from paper_conf_ppopp_li0yjl19_b200.batch import DeviceBatch  # noqa: E402
 
 NAMES = ["sched_rempty", "sched_budget", "prod_rfull", "prod_empty", "mma_rfull", "mma_tempty", "mma_full",
          "cprod_rfull", "cprod_cempty", "epi_rfull", "epi_tfull", "epi_cfull", "epi_store", "epi_tmem", "epi_math",
-         "total", "tiles"]
+         "total", "tiles", "prod_issue", "mma_issue", "epi_fencebar", "epi_stissue", "epi_loop"]
 WARPS = {"sched": 1, "prod": 1, "mma": 1, "cprod": 1, "epi": 8}
 
 ap = argparse.ArgumentParser()
@@ -47,7 +47,8 @@ v = buf.cpu().tolist()
 grid = min(plan.info()["n_blocks"], 148)
 total = v[NAMES.index("total")] / (12 * grid)
 print(f"{args.config} {args.policy}: {s.elapsed_time(e):.3f} ms, {total:.0f} cycles per CTA, tiles {v[16]}")
-for i, n in enumerate(NAMES[:15]):
+for i, n in enumerate(NAMES[:15] + NAMES[17:]):
+    i = NAMES.index(n)
     w = WARPS[n.split("_")[0]]
     cyc = v[i] / (w * grid)
     print(f"  {n:14s} {cyc / total * 100:6.1f}%")

@@ -243,3 +243,24 @@ def test_bind_then_exec_bound_repeatedly(dtype):
         check_bound(db, range(len(M)), SEED, "random", c_old=c_prev)
     with pytest.raises(vb.VbError):
         db.plan().exec_bound(db.alpha.data_ptr(), db.beta.data_ptr(), 0)   # never bound
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f16"])
+def test_rebind_alternating_buffers_never_uses_stale_descriptors(dtype):
+    # one plan, two batches with identical shapes in different arenas; re-bind back and forth
+    # (tensor maps are patched in place by the prep kernel) and check every result
+    M, N, K = vbinputs.config_sizes("C2")
+    M, N, K = M[:40], N[:40], K[:40]
+    dbs = [DeviceBatch(M, N, K, dtype), DeviceBatch(M, N, K, dtype)]
+    seeds = [11, 12]
+    for db, sd in zip(dbs, seeds):
+        db.fill(sd)
+    plan = dbs[0].plan()
+    c0 = [db.C.clone() for db in dbs]
+    for rnd in range(4):
+        i = rnd % 2
+        db = dbs[i]
+        db.C.copy_(c0[i])
+        db.run(plan)                   # bind (patch maps) + GEMM kernel
+        torch.cuda.synchronize()
+        check_batch(db, range(len(M)), seeds[i], "random")
