@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
 #include <stdarg.h>
+#include <stdlib.h>
 #include <stdio.h>
 #include <string.h>
 
@@ -121,7 +122,10 @@ static vb_status encode_2d(CUtensorMap *m, vb_dtype dt, void *addr, uint64_t inn
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = enc(m, t, 2, addr, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_of(swz_bytes),
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+#ifndef VB_L2PROMO
+#define VB_L2PROMO CU_TENSOR_MAP_L2_PROMOTION_L2_256B
+#endif
+                   VB_L2PROMO, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS)
     return fail(VB_ERR_INTERNAL, "cuTensorMapEncodeTiled failed (%d) dims %llu x %llu ld %llu box %u x %u", (int)r,
                 (unsigned long long)inner, (unsigned long long)outer, (unsigned long long)ld_elems, box_inner,
@@ -184,7 +188,7 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   const size_t o_ct = off;
   off = align_up(off + 256, 256);
   const size_t o_tm = off;
-  if (tc) off = align_up(off + (size_t)p->batch * 3 * 128, 256);
+  if (tc) off = align_up(off + (size_t)p->batch * kMapsPerGemm * 128, 256);
   p->ws_bytes = off;
   e = cudaMalloc(&p->d_ws, p->ws_bytes);
   if (e != cudaSuccess) {
@@ -213,17 +217,30 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
       if (M[i] == 0 || N[i] == 0) continue;
       const StrategyRow &s = p->table->rows[p->tiling.row[i]];
       const TcGeom g = tc_geom(s.BY, s.BX);
+      CUtensorMap *m = &maps[(size_t)kMapsPerGemm * i];
       vb_status st;
       if (K[i] > 0) {
-        st = encode_2d(&maps[3 * i + 0], p->dt, p->d_ws, (uint64_t)K[i], (uint64_t)M[i], (uint64_t)lda[i], 64,
+        st = encode_2d(&m[MAP_A], p->dt, p->d_ws, (uint64_t)K[i], (uint64_t)M[i], (uint64_t)lda[i], 64,
                        (uint32_t)s.BY, 128);
         if (st != VB_OK) return st;
-        st = encode_2d(&maps[3 * i + 1], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)K[i], (uint64_t)ldb[i],
+        if (M[i] % s.BY) {   // last row-tile: box of the remaining rows only (rounded up to 8)
+          const uint32_t rows = (uint32_t)((M[i] % s.BY + 7) / 8 * 8);
+          st = encode_2d(&m[MAP_A_TAIL], p->dt, p->d_ws, (uint64_t)K[i], (uint64_t)M[i], (uint64_t)lda[i], 64, rows,
+                         128);
+          if (st != VB_OK) return st;
+        }
+        st = encode_2d(&m[MAP_B], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)K[i], (uint64_t)ldb[i],
                        (uint32_t)(g.b_swz / 2), 64, g.b_swz);
         if (st != VB_OK) return st;
+        if (K[i] % 64) {     // last k-block: box of the remaining K rows only (rounded up to 16)
+          const uint32_t rows = (uint32_t)((K[i] % 64 + 15) / 16 * 16);
+          st = encode_2d(&m[MAP_B_TAIL], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)K[i], (uint64_t)ldb[i],
+                         (uint32_t)(g.b_swz / 2), rows, g.b_swz);
+          if (st != VB_OK) return st;
+        }
       }
-      // C box = one epilogue warp's sub-box: c_cols x BY/4 rows
-      st = encode_2d(&maps[3 * i + 2], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)M[i], (uint64_t)ldc[i],
+      // C box = one epilogue quarter's sub-box: c_cols x BY/4 rows
+      st = encode_2d(&m[MAP_C], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)M[i], (uint64_t)ldc[i],
                      (uint32_t)g.c_cols, (uint32_t)(s.BY / 4), g.c_swz);
       if (st != VB_OK) return st;
     }
@@ -239,6 +256,7 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
                              const Schedule &sch) {
   p->block_ptr = sch.block_ptr;
   p->slots.resize(sch.slot_tile.size());
+
   for (size_t s = 0; s < sch.slot_tile.size(); ++s) {
     const TileRec &t = tiles[(size_t)sch.slot_tile[s]];
     if (t.y > 0xFFFF || t.x > 0xFFFF) return fail(VB_ERR_INVALID_ARG, "tile index above 65535");
@@ -276,6 +294,7 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
       // last C chunk of this tile ends inside a 16-byte granule of the row -> direct stores
       const int last_chunk_end = d.n0 + s.BX;
       d.flags = (uint16_t)(((g.N & 7) != 0 && last_chunk_end > g.N && d.n0 < g.N) ? 1 : 0);
+      if (g.K % 64) d.flags |= (uint16_t)(((g.K % 64 + 15) / 16) << 8);   // MMA K-steps of the last k-block
       (void)geo;
     }
   }

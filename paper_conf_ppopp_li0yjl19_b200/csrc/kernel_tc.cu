@@ -2,22 +2,25 @@
 // engine's work lists (Fig. 7, P294-312) with TMA-staged operands and tcgen05
 // tensor-core MMA accumulating in TMEM.
 //
-// One CTA per SM (grid = min(Block_NUM, #SMs)), 8 warps:
+// One CTA per SM (grid = min(Block_NUM, #SMs)), 16 warps:
 //   warp 0      scheduler: claims the next block (work list) with an atomic (one block
 //               ahead), loads its tile descriptors (one 32-byte record per tile, lanes in
-//               parallel) and alpha/beta, and publishes them in a 32-entry smem tile ring.
-//   warp 1      A/B producer: streams each tile's k-blocks (A: BY x 64, B: 64 x BX) with TMA
-//               into a PAGED ring (18 pages of 8 KB): a k-block takes only the pages it needs
-//               (2 for a 64x32 tile, 6 for 128x256), so small tiles keep up to 9 k-blocks in
-//               flight — the paper's ILP concern for small K (P151, P259) mapped to TMA depth.
-//   warp 2      TMEM allocator + MMA issuer: one thread issues tcgen05.mma (M = BY, N = BX,
-//               K = 16) into one of two 256-column fp32 accumulators.
-//   warp 3      C producer: TMA-loads C_old chunks (BY x 64) into a 4-slot ring when
-//               beta != 0 (C is never read when beta == 0, reading C-16).
-//   warps 4-7   epilogue: tcgen05.ld (warp w owns TMEM lanes 32*(w%4)..), C = alpha*acc +
-//               beta*C_old in fp32, RNE to bf16/fp16, write back into the swizzled smem chunk,
-//               TMA store (completion deferred by one chunk); the accumulator is released
-//               to the MMA warp as soon as its last columns are in registers.
+//               parallel) and alpha/beta into a 32-entry smem tile ring, prefetches the tiles'
+//               tensor maps; lookahead is bounded in k-blocks so the GPU works on a short
+//               window of GEMMs at a time (L2 reuse of A/B).
+//   warp 1      TMEM owner + MMA issuer: one thread issues tcgen05.mma (M = BY, N = BX,
+//               K = 16) into an accumulator ring of 512 TMEM columns (up to 8 tiles in flight).
+//   warps 2-3   C_old producers: TMA-load C_old chunks (BY x 64) per epilogue quarter into a
+//               4-slot ring when beta != 0 (C is never read when beta == 0, reading C-16).
+//   warps 4-7   A/B producers: stream each tile's k-blocks (A: BY x 64, B: 64 x BX) with TMA
+//               into a PAGED ring (18 pages of 8 KB; a k-block takes 2 pages for 64x32 ... 6
+//               for 128x256, so small tiles keep up to 9 k-blocks in flight — the paper's ILP
+//               concern for small K, P151/P259, as TMA depth).  One thread issues only ~1 TMA
+//               box per 250 cycles, so four warps split every k-block's boxes.
+//   warps 8-15  epilogue: warps 8+q and 12+q own TMEM lane quarter q and split each chunk's
+//               columns; tcgen05.ld, C = alpha*acc + beta*C_old in fp32, RNE to bf16/fp16 in
+//               the swizzled smem chunk, TMA store of the quarter's sub-box (completion
+//               deferred one chunk); the accumulator is released after its last tcgen05.ld.
 // The paper's "unified thread structure" (P181) becomes a runtime MMA instruction descriptor
 // per tile, so one kernel serves every strategy of the table.
 #include <cuda.h>
@@ -32,7 +35,12 @@
 namespace vb {
 namespace tck {
 
-constexpr int kThreads = 384;              // 4 role warps + 8 epilogue warps
+constexpr int kThreads = 512;              // 16 warps: see the role table in the header comment
+#ifndef VB_NPROD
+#define VB_NPROD 4
+#endif
+constexpr int kProducers = VB_NPROD;       // A/B TMA issuing warps (one thread issues ~1 box / 250 cycles)
+constexpr int kCProducers = 2;             // C_old TMA issuing warps
 constexpr int kBK = 64;                    // bf16 elements per k-block = one 128-B swizzle row
 constexpr int kPageBytes = 8192;
 #ifndef VB_PAGES
@@ -55,7 +63,7 @@ constexpr int kAccUnit = 32;               // TMEM accumulator ring granularity 
 constexpr int kAccUnits = kTmemCols / kAccUnit;
 constexpr int kAcc = 8;                    // accumulators in flight (ring entries)
 constexpr int kEpiWarps = 8;               // two per TMEM lane quarter, splitting each chunk's columns
-constexpr uint32_t kRingConsumers = 1 + 1 + 1 + kEpiWarps;   // producer, MMA, C producer, epilogue warps
+constexpr uint32_t kRingConsumers = kProducers + 1 + kCProducers + kEpiWarps;
 
 struct TileInfo {          // one tile ring entry (48 bytes)
   TileDesc d;
@@ -70,7 +78,7 @@ struct Shared {
   uint64_t cfull[kCSlots], cempty[kCSlots];
   uint64_t rfull[kRing], rempty[kRing];
   int32_t slot_page[kSlots];
-  int32_t slot_pages[kSlots];   // producer-private: pages charged to each k-block in flight
+  int32_t slot_pages[kProducers][kSlots];   // per producer replica: pages charged per k-block
   int32_t acc_take[kAcc];       // MMA-private: TMEM units charged to each accumulator in flight
   uint32_t tmem_base;
   volatile uint32_t prod_kb;    // k-blocks (>= 1 per tile) the A/B producer has finished issuing
@@ -215,7 +223,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       ptx::mbar_init(&sh->tempty[i], kEpiWarps);
     }
     for (int i = 0; i < kCSlots; ++i) {
-      ptx::mbar_init(&sh->cfull[i], 1);
+      ptx::mbar_init(&sh->cfull[i], kCProducers);
       ptx::mbar_init(&sh->cempty[i], 4);   // one arrival per lane quarter (its storing warp)
     }
     for (int i = 0; i < kRing; ++i) {
@@ -225,7 +233,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     sh->prod_kb = 0u;
     ptx::fence_mbar_init();
   }
-  if (warp == 2) ptx::tmem_alloc(&sh->tmem_base, kTmemCols);
+  if (warp == 1) ptx::tmem_alloc(&sh->tmem_base, kTmemCols);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
@@ -264,12 +272,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           const TileDesc d = p.tiles[base + lane];
           kb = max(d.kblocks, 1);
           // warm the TMA descriptor cache for the tile's maps well before the producers use them
-          const uint8_t *maps = tmaps + (size_t)d.gemm * 384;
+          const uint8_t *maps = tmaps + (size_t)d.gemm * (kMapsPerGemm * 128);
           if (d.kblocks > 0) {
-            ptx::prefetch_tmap(maps);
-            ptx::prefetch_tmap(maps + 128);
+            ptx::prefetch_tmap(maps + MAP_A * 128);
+            ptx::prefetch_tmap(maps + MAP_B * 128);
           }
-          ptx::prefetch_tmap(maps + 256);
+          ptx::prefetch_tmap(maps + MAP_C * 128);
           const float al = p.alpha[d.gemm], be = p.beta[d.gemm];
           const uint32_t tt = t + lane;
           const int e = (int)(tt % kRing);
@@ -293,12 +301,18 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       sh->ring[e].d.gemm = -1;
       ptx::mbar_arrive(&sh->rfull[e]);
     }
-  } else if (warp == 1) {
-    // ================================================================ A/B TMA producer
-    if (lane == 0) {
+  } else if (warp >= 4 && warp < 8) {
+    // ================================================================ A/B TMA producers
+    // kProducers warps run the same deterministic page allocator over the same tile sequence
+    // (so they agree on every k-block's pages without talking) and split each k-block's TMA
+    // boxes round-robin: one thread can issue only ~1 box per 250 cycles.  Producer 0 alone
+    // arms the full barrier (arrive + expect_tx of the k-block's total bytes), publishes the
+    // k-block's page, and reports progress to the scheduler.
+    const int pid = warp - 4;
+    if (lane == 0 && pid < kProducers) {
       int re = 0, slot = 0, head = 0, oldest = 0, inflight = 0, free_pages = kPages;
-      uint32_t rph = 0, sph = 0, ophase = 0;
-      int32_t *slot_pages = sh->slot_pages;
+      uint32_t rph = 0, sph = 0, ophase = 0, kbg = 0;
+      int32_t *slot_pages = sh->slot_pages[pid];
       for (;;) {
         VB_TWAIT(T_PROD_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
         const TileInfo ti = sh->ring[re];
@@ -306,50 +320,72 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         advance(re, rph, kRing);
         if (ti.d.gemm < 0) break;
         if (ti.d.kblocks == 0) {
-          sh->prod_kb = sh->prod_kb + 1u;
+          if (pid == 0) sh->prod_kb = sh->prod_kb + 1u;
           continue;
         }
         const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
         const TcGeom geo = tc_geom(BY, BX);
-        const uint8_t *mapA = tmaps + (size_t)ti.d.gemm * 384;
-        const uint8_t *mapB = mapA + 128;
-        const int a_bytes = BY * kBK * 2, b_bytes = BX * kBK * 2;
-        const int a_pages = a_bytes / kPageBytes;
-        const int need = a_pages + (b_bytes + kPageBytes - 1) / kPageBytes;
-        for (int kb = 0; kb < ti.d.kblocks; ++kb) {
+        const uint8_t *maps = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128);
+        // out-of-bounds box rows cost L2 bandwidth even though TMA zero-fills them: the last
+        // row-tile uses the row-tail map, the last k-block the K-tail map, and B boxes that lie
+        // entirely past N are not loaded (their MMA columns are discarded by the epilogue)
+        const int a_rows = min(BY, ti.d.M - ti.d.m0);
+        const bool a_tail = a_rows < BY;
+        const uint8_t *mapA = maps + (a_tail ? MAP_A_TAIL : MAP_A) * 128;
+        const int a_box_rows = a_tail ? (a_rows + 7) / 8 * 8 : BY;
+        const int b_boxes = min(geo.b_boxes, (ti.d.N - ti.d.n0 + geo.b_swz / 2 - 1) / (geo.b_swz / 2));
+        const int ksteps_last = (ti.d.flags >> 8) & 7;
+        const int a_pages = BY * kBK * 2 / kPageBytes;
+        const int need = a_pages + (BX * kBK * 2 + kPageBytes - 1) / kPageBytes;
+        for (int kb = 0; kb < ti.d.kblocks; ++kb, ++kbg) {
           int start = head, take = need;
           if (start + need > kPages) {          // never wrap a k-block around the ring end
             take += kPages - start;
             start = 0;
           }
-          while (free_pages < take || inflight == kSlots) {
-            // reclaim the oldest k-block in flight once the MMA has consumed it
-            VB_TWAIT(T_PROD_EMPTY, ptx::mbar_wait(&sh->empty[oldest], ophase));
-            free_pages += slot_pages[oldest];
-            --inflight;
-            advance(oldest, ophase, kSlots);
+          {
+            VB_T0();
+            while (free_pages < take || inflight == kSlots) {
+              // reclaim the oldest k-block in flight once the MMA has consumed it
+              ptx::mbar_wait(&sh->empty[oldest], ophase);
+              free_pages += slot_pages[oldest];
+              --inflight;
+              advance(oldest, ophase, kSlots);
+            }
+            VB_TADD(T_PROD_EMPTY);
           }
           slot_pages[slot] = take;
           free_pages -= take;
           ++inflight;
           head = start + need;
           if (head == kPages) head = 0;
-          sh->slot_page[slot] = start;
-          VB_T0();
-          ptx::mbar_arrive_expect_tx(&sh->full[slot], (uint32_t)(a_bytes + b_bytes));
+          const bool k_tail = (kb == ti.d.kblocks - 1) && ksteps_last != 0;
+          const int b_rows = k_tail ? ksteps_last * 16 : kBK;
+          const uint8_t *mapB = maps + (k_tail ? MAP_B_TAIL : MAP_B) * 128;
           uint8_t *sa = pages + (size_t)start * kPageBytes;
           uint8_t *sb = sa + (size_t)a_pages * kPageBytes;
-          ptx::tma_load_2d(sa, mapA, &sh->full[slot], kb * kBK, ti.d.m0);
-          for (int j = 0; j < geo.b_boxes; ++j)
-            ptx::tma_load_2d(sb + j * kBK * geo.b_swz, mapB, &sh->full[slot], ti.d.n0 + j * (geo.b_swz / 2), kb * kBK);
+          VB_T0();
+          if (pid == 0) {
+            sh->slot_page[slot] = start;
+            ptx::mbar_arrive_expect_tx(&sh->full[slot],
+                                       (uint32_t)(a_box_rows * kBK * 2 + b_boxes * b_rows * geo.b_swz));
+          }
+          // box 0 = A, boxes 1..b_boxes = B; box i goes to producer (i + kbg) % kProducers
+          for (int i = (int)((pid - kbg) % kProducers + kProducers) % kProducers; i <= b_boxes; i += kProducers) {
+            if (i == 0)
+              ptx::tma_load_2d(sa, mapA, &sh->full[slot], kb * kBK, ti.d.m0);
+            else
+              ptx::tma_load_2d(sb + (i - 1) * kBK * geo.b_swz, mapB, &sh->full[slot],
+                               ti.d.n0 + (i - 1) * (geo.b_swz / 2), kb * kBK);
+          }
           VB_TADD(T_PROD_ISSUE);
           advance(slot, sph, kSlots);
-          sh->prod_kb = sh->prod_kb + 1u;
+          if (pid == 0) sh->prod_kb = sh->prod_kb + 1u;
         }
       }
     }
-  } else if (warp == 2) {
-    // ================================================================ MMA issuer
+  } else if (warp == 1) {
+    // ================================================================ MMA issuer (+ TMEM owner)
     if (lane == 0) {
       int re = 0, slot = 0, oldest = 0, free_units = kAccUnits, inflight = 0;
       uint32_t rph = 0, sph = 0, t = 0, ophase = 0;
@@ -394,14 +430,20 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           VB_T0();
           const uint32_t sa = ptx::smem_u32(pages + (size_t)sh->slot_page[slot] * kPageBytes);
           const uint32_t sb = sa + a_bytes;
+          const int ksteps = (kb == ti.d.kblocks - 1 && ((ti.d.flags >> 8) & 7)) ? ((ti.d.flags >> 8) & 7) : kBK / 16;
 #pragma unroll
           for (int kk = 0; kk < kBK / 16; ++kk) {
+            if (kk >= ksteps) break;          // K tail: the B rows past the last step are not loaded
             // A: K-major, 128-B swizzle, 8-row atoms 1024 B apart; K step of 16 = +32 B.
             const uint64_t adesc = ptx::smem_desc(sa + kk * 32, 16, 1024, 2);
             // B: MN-major, b_swz swizzle; 8-row (K) atoms 8*b_swz apart (SBO), MN blocks of
             // b_swz/2 elements 64*b_swz apart (LBO); K step of 16 rows = +16*b_swz bytes.
             const uint64_t bdesc = ptx::smem_desc(sb + kk * 16 * geo.b_swz, kBK * geo.b_swz, 8 * geo.b_swz, blayout);
+#ifndef VB_EXP_NOMMA
             ptx::mma_f16_ss(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
+#else
+            (void)adesc; (void)bdesc; (void)idesc; (void)d_tmem;
+#endif
           }
           ptx::mma_commit(&sh->empty[slot]);      // frees the k-block's pages when the MMAs retire
           VB_TADD(T_MMA_ISSUE);
@@ -410,8 +452,10 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         ptx::mma_commit(&sh->tfull[e]);           // accumulator ready for the epilogue
       }
     }
-  } else if (warp == 3) {
-    // ================================================================ C_old producer
+  } else if (warp == 2 || warp == 3) {
+    // ================================================================ C_old producers
+    // warp 2 loads the sub-boxes of lane quarters 0-1, warp 3 those of quarters 2-3
+    const int cid = warp - 2;
     if (lane == 0) {
       int re = 0, cs = 0;
       uint32_t rph = 0, cph = 0;
@@ -424,17 +468,17 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         if (ti.d.gemm < 0) break;
         const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
         const TcGeom geo = tc_geom(BY, BX);
-        const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * 384 + 256;
+        const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C * 128;
         const bool load = ti.beta != 0.f;
         for (int ch = 0; ch < geo.c_chunks; ++ch) {
           VB_TWAIT(T_CPROD_CEMPTY, ptx::mbar_wait(&sh->cempty[cs], cph ^ 1u));
           if (load) {
-            // the C map's box is one epilogue warp's sub-box (BY/4 rows); skip rows >= M
+            // the C map's box is one epilogue quarter's sub-box (BY/4 rows); skip rows >= M
             const int rows_w = BY / 4;
             int nsub = 0;
-            for (int w = 0; w < 4; ++w) nsub += (ti.d.m0 + w * rows_w < ti.d.M) ? 1 : 0;
+            for (int w = 2 * cid; w < 2 * cid + 2; ++w) nsub += (ti.d.m0 + w * rows_w < ti.d.M) ? 1 : 0;
             ptx::mbar_arrive_expect_tx(&sh->cfull[cs], (uint32_t)(nsub * rows_w * geo.c_cols * 2));
-            for (int w = 0; w < nsub; ++w)
+            for (int w = 2 * cid; w < 2 * cid + nsub; ++w)
               ptx::tma_load_2d_hint(cbuf + (size_t)cs * kCSlotBytes + w * rows_w * geo.c_swz, mapC, &sh->cfull[cs],
                                     ti.d.n0 + ch * geo.c_cols, ti.d.m0 + w * rows_w, c_policy);
           } else {
@@ -446,12 +490,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     }
   } else {
     // ================================================================ epilogue (8 warps)
-    // Warps 4+q and 8+q share TMEM lane quarter q (tile rows r0 .. r0+BY/4-1) and split each
+    // Warps 8+q and 12+q share TMEM lane quarter q (tile rows r0 .. r0+BY/4-1) and split each
     // chunk's columns in halves.  The pair meets on a 64-thread named barrier per chunk, then
-    // warp 4+q TMA-stores the quarter's sub-box itself: no barrier spans all epilogue warps,
-    // and TMEM loads of the next chunk are issued before the current one is processed.
+    // warp 8+q TMA-stores the quarter's sub-box itself: no barrier spans all epilogue warps.
     const int q = warp & 3;
-    const int half = (warp - 4) >> 2;
+    const int half = (warp - 8) >> 2;
     const bool storer = half == 0;
     const uint64_t c_policy = ptx::policy_evict_first();
     int re = 0, cs = 0, pending = -1;
@@ -466,7 +509,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       if (ti.d.gemm < 0) break;
       const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
       const TcGeom geo = tc_geom(BY, BX);
-      const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * 384 + 256;
+      const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C * 128;
       const int e = (int)(t % kAcc);
       const uint32_t aph = (t / kAcc) & 1u;
       ++t;
@@ -571,25 +614,19 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         advance(cs, cph, kCSlots);
       };
 
-      uint32_t a0[32], a1[32];
+      uint32_t a0[32];
       const int nch = geo.c_chunks;
-      if (has_acc) {
-        tload(0, a0);
-      } else {
+      if (!has_acc) {
 #pragma unroll
-        for (int i = 0; i < 32; ++i) a0[i] = a1[i] = 0u;   // K == 0: C = beta * C
+        for (int i = 0; i < 32; ++i) a0[i] = 0u;   // K == 0: C = beta * C
       }
-      for (int ch = 0; ch < nch; ch += 2) {
-        if (has_acc) VB_TWAIT(T_EPI_TMEM, ptx::tmem_ld_wait());
-        if (has_acc && ch + 1 < nch) tload(ch + 1, a1);
-        if (ch + 1 >= nch) release_acc();
-        process(ch, a0);
-        if (ch + 1 < nch) {
-          if (has_acc) VB_TWAIT(T_EPI_TMEM, ptx::tmem_ld_wait());
-          if (has_acc && ch + 2 < nch) tload(ch + 2, a0);
-          if (ch + 2 >= nch) release_acc();
-          process(ch + 1, a1);
+      for (int ch = 0; ch < nch; ++ch) {
+        if (has_acc) {
+          tload(ch, a0);
+          VB_TWAIT(T_EPI_TMEM, ptx::tmem_ld_wait());
         }
+        if (ch + 1 == nch) release_acc();
+        process(ch, a0);
       }
 #ifdef VB_TRACE
       tr[T_EPI_LOOP] += clock64() - _tile_t0;
@@ -607,7 +644,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
-  if (warp == 2) ptx::tmem_dealloc(tmem_base, kTmemCols);
+  if (warp == 1) ptx::tmem_dealloc(tmem_base, kTmemCols);
   // The last CTA to finish resets the work-list counter, so back-to-back launches of the
   // same bound plan need no reset kernel.  Every CTA fetched past n_blocks before getting here.
   if (threadIdx.x == 0) {
@@ -633,12 +670,17 @@ __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
     counter[0] = 0;
     counter[1] = 0;
   }
-  if (i >= batch * 3) return;
-  const int g = i / 3, w = i % 3;
+  if (i >= batch * kMapsPerGemm) return;
+  const int g = i / kMapsPerGemm, w = i % kMapsPerGemm;
   const GemmParam gp = gemms[g];
   if (gp.M <= 0 || gp.N <= 0) return;
-  if (w < 2 && gp.K <= 0) return;
-  const void *ptr = w == 0 ? A[g] : (w == 1 ? B[g] : static_cast<const void *>(C[g]));
+  const int BY = (gp.row >> 8) & 0xFF;
+  if (w != MAP_C && gp.K <= 0) return;
+  if (w == MAP_A_TAIL && gp.M % BY == 0) return;        // map not encoded
+  if (w == MAP_B_TAIL && gp.K % 64 == 0) return;
+  const void *ptr = (w == MAP_A || w == MAP_A_TAIL) ? A[g]
+                    : (w == MAP_B || w == MAP_B_TAIL) ? B[g]
+                                                      : static_cast<const void *>(C[g]);
   ptx::tmap_replace_address(tmaps + (size_t)i * 128, ptr);
   ptx::tmap_release();
 }
@@ -657,7 +699,7 @@ cudaError_t tc_configure() {
 
 cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
                            const GemmParam *gemms, int batch, int32_t *counter, cudaStream_t stream) {
-  const int n = batch * 3;
+  const int n = batch * kMapsPerGemm;
   tck::vb_tc_prep<<<n > 0 ? (n + 255) / 256 : 1, 256, 0, stream>>>(tmaps, A, B, C, gemms, batch, counter);
   return cudaGetLastError();
 }

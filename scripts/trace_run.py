@@ -19,13 +19,13 @@ from paper_conf_ppopp_li0yjl19_b200.batch import DeviceBatch  # noqa: E402
 NAMES = ["sched_rempty", "sched_budget", "prod_rfull", "prod_empty", "mma_rfull", "mma_tempty", "mma_full",
          "cprod_rfull", "cprod_cempty", "epi_rfull", "epi_tfull", "epi_cfull", "epi_store", "epi_tmem", "epi_math",
          "total", "tiles", "prod_issue", "mma_issue", "epi_fencebar", "epi_stissue", "epi_loop"]
-WARPS = {"sched": 1, "prod": 1, "mma": 1, "cprod": 1, "epi": 8}
+WARPS = {"sched": 1, "prod": 1, "mma": 1, "cprod": 1, "epi": 8, "cprod": 2, "prod": 4}
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C5")
 ap.add_argument("--policy", default="threshold")
 args = ap.parse_args()
-assert "trace" in nv.LIB_PATH, "set VB_LIB to the trace build"
+assert "trace" in nv.LIB_PATH, "set VB_LIB to a trace build"
 info = vbinputs.CONFIGS[args.config]
 M, N, K = vbinputs.config_sizes(args.config)
 db = DeviceBatch(M, N, K, info["dtype"])
@@ -45,7 +45,7 @@ torch.cuda.synchronize()
 nv.lib.vb_debug_set_trace(None)
 v = buf.cpu().tolist()
 grid = min(plan.info()["n_blocks"], 148)
-total = v[NAMES.index("total")] / (12 * grid)
+total = v[NAMES.index("total")] / (16 * grid)
 print(f"{args.config} {args.policy}: {s.elapsed_time(e):.3f} ms, {total:.0f} cycles per CTA, tiles {v[16]}")
 for i, n in enumerate(NAMES[:15] + NAMES[17:]):
     i = NAMES.index(n)
