@@ -76,15 +76,19 @@ def check_plan_invariants(p: Plan, Ms, Ns, Ks, policy: int, theta: int) -> None:
             assert 1 <= len(blk) <= 2
             if len(blk) == 2:
                 assert Kt[blk[0]] <= Kt[blk[1]] < theta
+    # pair (2-SM) tiles come first and are batched separately from the single tiles
+    n_pair = sum(1 for t in p.tiles if p.table.rows[p.tiling.rows[t.gemm]].ctas == 2)
+    assert all(p.table.rows[p.tiling.rows[t.gemm]].ctas == 2 for t in p.tiles[:n_pair])
+    for blk in p.blocks:
+        assert all(t < n_pair for t in blk) or all(t >= n_pair for t in blk), "homogeneous blocks"
     if policy == POLICY_THRESHOLD:
         # a block with more than one tile was opened in fill mode: its K-sum reached θ
-        # only with its last tile (or tiles ran out at the end of the list)
-        last = len(p.blocks) - 1
-        for b, blk in enumerate(p.blocks):
+        # only with its last tile (or its partition's tiles ran out)
+        for blk in p.blocks:
             if len(blk) > 1:
                 ks = [Kt[t] for t in blk]
                 assert sum(ks[:-1]) < theta
-                assert sum(ks) >= theta or b == last or blk[-1] == n_tiles - 1
+                assert sum(ks) >= theta or blk[-1] in (n_pair - 1, n_tiles - 1)
     # tiler trace: each round's strategy per GEMM is at least as late in priority order
     # (tile area never shrinks); the final strategy fits the GEMM unless nothing fits (C-1, C-4)
     tr = p.tiling.trace

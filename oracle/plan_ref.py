@@ -22,6 +22,7 @@ class Strategy:
     BY: int      # tile rows    (along M)
     BX: int      # tile columns (along N)
     BK: int      # K step of one main-loop iteration
+    ctas: int = 1  # CTAs executing one tile (2 = tcgen05 cta_group::2 pair tile)
 
 
 @dataclass(frozen=True)
@@ -56,13 +57,14 @@ B200_F32 = Table("b200_ffma", V100.rows, versions=(256, 128), tlp_threshold=1310
 
 # B200 tcgen05 (bf16/fp16) profile: C-tile shapes sized for tcgen05.mma
 # (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16), plus the skinny shapes
-# 128x32 and 64x256.  One kernel "version" with T = 256 threads (8 warps).  Availability
+# 128x32 and 64x256, plus 2-SM pair tiles 256x{64,128,256} (ctas = 2, cta_group::2).  One kernel "version" with T = 256 threads (8 warps).  Availability
 # floor (C-1b): a GEMM shorter than 64 rows still occupies a 64-row MMA, so strategies are
 # tested against max(M, 64) and max(N, 32).
 B200_TC = Table("b200_tcgen05", (
     Strategy("s", 64, 32, 64), Strategy("n", 128, 32, 64), Strategy("m", 64, 64, 64), Strategy("t", 128, 64, 64),
     Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("x", 64, 256, 64),
-    Strategy("h", 128, 256, 64)),
+    Strategy("h", 128, 256, 64), Strategy("T2", 256, 64, 64, 2), Strategy("L2", 256, 128, 64, 2),
+    Strategy("H2", 256, 256, 64, 2)),
     versions=(256,), tlp_threshold=4 * 148 * 256, theta=512, min_BY=64, min_BX=32)
 
 TABLES = {1: V100, 2: B200_F32, 3: B200_TC}
@@ -76,7 +78,7 @@ def tlp(Ms, Ns, rows: Sequence[int], table: Table, T: int) -> int:
     total = 0
     for M, N, r in zip(Ms, Ns, rows):
         s = table.rows[r]
-        total += ceil(M / s.BY) * ceil(N / s.BX)
+        total += ceil(M / s.BY) * ceil(N / s.BX) * s.ctas      # a pair tile occupies two CTAs
     return total * T
 
 
@@ -90,7 +92,7 @@ class TilingResult:
         return [table.strategy_id(r, self.T) for r in self.rows]
 
 
-def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None) -> TilingResult:
+def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None, pairs_allowed: bool = True) -> TilingResult:
     """The three steps and two exceptions of P249–253.
 
     1. Per GEMM, a priority queue of the strategies with BY <= M and BX <= N (C-1; the
@@ -107,6 +109,8 @@ def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None) -> TilingR
     """
     thr = table.tlp_threshold if threshold is None else threshold
     order = table.order()
+    if not pairs_allowed:                                             # C-7b
+        order = [r for r in order if table.rows[r].ctas == 1]
     queues = []
     for M, N in zip(Ms, Ns):
         mf, nf = max(M, table.min_BY), max(N, table.min_BX)           # C-1b (0 for the paper's tables)
@@ -256,21 +260,43 @@ class Plan:
     enc: Encoded
 
 
+PAIR_MIN_AI = 128     # flop per compulsory byte (reading C-7b)
+
+
+def pairs_allowed(Ms, Ns, Ks, es: int = 2) -> bool:
+    """Reading C-7b: the 2-SM pair version (cta_group::2) is offered only to batches whose
+    arithmetic intensity 2*sum(MNK) / sum(es*(MK + KN) + 2*es*MN) is at least 128 flop/B, i.e.
+    batches near the compute side of the B200 ridge (~265 flop/B); memory-bound batches keep
+    the 1-SM version so that their compute- and memory-heavy tiles overlap in one kernel."""
+    flops = sum(2 * m * n * k for m, n, k in zip(Ms, Ns, Ks))
+    nbytes = sum(es * (m * k + k * n) + 2 * es * m * n for m, n, k in zip(Ms, Ns, Ks) if m > 0 and n > 0)
+    return flops >= PAIR_MIN_AI * nbytes and nbytes > 0
+
+
 def plan(Ms, Ns, Ks, table: Table, policy: int = POLICY_THRESHOLD,
-         tlp_threshold: int | None = None, theta: int | None = None) -> Plan:
+         tlp_threshold: int | None = None, theta: int | None = None, es: int = 2) -> Plan:
     thr = table.tlp_threshold if tlp_threshold is None else tlp_threshold
     th = table.theta if theta is None else theta
     Ms = [int(v) for v in Ms]; Ns = [int(v) for v in Ns]; Ks = [int(v) for v in Ks]
-    tr = tiling_engine(Ms, Ns, table, thr)
-    tiles = enumerate_tiles(Ms, Ns, Ks, tr.rows, table)
-    if policy == POLICY_THRESHOLD:
-        blocks = threshold_batching(tiles, tr.T, thr, th)
-    elif policy == POLICY_BINARY:
-        blocks = binary_batching(tiles, th)
-    elif policy == POLICY_NONE:
-        blocks = no_batching(tiles)
-    else:
-        raise ValueError(policy)
+    tr = tiling_engine(Ms, Ns, table, thr, pairs_allowed(Ms, Ns, Ks, es))
+    all_tiles = enumerate_tiles(Ms, Ns, Ks, tr.rows, table)
+    # 2-SM pair tiles run in their own (cluster) kernel: the batching engine packs the pair
+    # tiles and the single tiles separately (each keeps enumeration order); pair blocks first.
+    is_pair = [table.rows[tr.rows[t.gemm]].ctas == 2 for t in all_tiles]
+    tiles = [t for t, pp in zip(all_tiles, is_pair) if pp] + [t for t, pp in zip(all_tiles, is_pair) if not pp]
+    n_pair = sum(is_pair)
+    blocks = []
+    for lo, hi in ((0, n_pair), (n_pair, len(tiles))):
+        part = tiles[lo:hi]
+        if policy == POLICY_THRESHOLD:
+            b = threshold_batching(part, tr.T, thr, th)
+        elif policy == POLICY_BINARY:
+            b = binary_batching(part, th)
+        elif policy == POLICY_NONE:
+            b = no_batching(part)
+        else:
+            raise ValueError(policy)
+        blocks += [[lo + i for i in blk] for blk in b]
     enc = encode(tiles, blocks, tr.ids(table))
     return Plan(table, tr, tiles, blocks, enc)
 

@@ -23,7 +23,7 @@ namespace vb {
 cudaError_t launch_f32(const F32Args &args, int n_blocks, int version_T, cudaStream_t stream);
 cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
                            const GemmParam *gemms, int batch, int32_t *counter, cudaStream_t stream);
-cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, cudaStream_t stream);
+cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, cudaStream_t stream);
 cudaError_t tc_configure();
 size_t tc_smem_bytes();
 cudaError_t launch_fill(int dt, int batch, const int32_t *rows, const int32_t *cols, const int32_t *ld,
@@ -74,7 +74,8 @@ struct vb_plan {
   TileDesc *d_tiles = nullptr;      // tensor-core path: one record per slot
   std::vector<TileDesc> tiles;
   uint8_t *d_tmaps = nullptr;
-  int32_t *d_counter = nullptr;     // [0] work-list counter, [1] finished-CTA counter
+  int32_t *d_counter = nullptr;     // pair kernel [0] work-list, [1] finished CTAs; 1-SM kernel [2], [3]
+  int n_pair_blocks = 0;            // blocks [0, n_pair_blocks) hold 2-SM pair tiles
   int sm_count = 0;
   const void *const *bound_A = nullptr;   // last vb_plan_bind
   const void *const *bound_B = nullptr;
@@ -216,32 +217,35 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
     for (int i = 0; i < p->batch; ++i) {
       if (M[i] == 0 || N[i] == 0) continue;
       const StrategyRow &s = p->table->rows[p->tiling.row[i]];
-      const TcGeom g = tc_geom(s.BY, s.BX);
+      // per-CTA view: a pair tile gives each CTA BY/2 rows of A and BX/2 columns of B
+      const int BYc = s.BY / s.ctas;
+      const TcGeom g = tc_geom(BYc, s.BX);                 // C chunks span the full BX
+      const TcGeom gb = tc_geom(BYc, s.BX / s.ctas);       // B boxes of this CTA's half
       CUtensorMap *m = &maps[(size_t)kMapsPerGemm * i];
       vb_status st;
       if (K[i] > 0) {
         st = encode_2d(&m[MAP_A], p->dt, p->d_ws, (uint64_t)K[i], (uint64_t)M[i], (uint64_t)lda[i], 64,
-                       (uint32_t)s.BY, 128);
+                       (uint32_t)BYc, 128);
         if (st != VB_OK) return st;
-        if (M[i] % s.BY) {   // last row-tile: box of the remaining rows only (rounded up to 8)
-          const uint32_t rows = (uint32_t)((M[i] % s.BY + 7) / 8 * 8);
+        if (M[i] % BYc) {   // last row-tile: box of the remaining rows only (rounded up to 8)
+          const uint32_t rows = (uint32_t)((M[i] % BYc + 7) / 8 * 8);
           st = encode_2d(&m[MAP_A_TAIL], p->dt, p->d_ws, (uint64_t)K[i], (uint64_t)M[i], (uint64_t)lda[i], 64, rows,
                          128);
           if (st != VB_OK) return st;
         }
         st = encode_2d(&m[MAP_B], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)K[i], (uint64_t)ldb[i],
-                       (uint32_t)(g.b_swz / 2), 64, g.b_swz);
+                       (uint32_t)(gb.b_swz / 2), 64, gb.b_swz);
         if (st != VB_OK) return st;
         if (K[i] % 64) {     // last k-block: box of the remaining K rows only (rounded up to 16)
           const uint32_t rows = (uint32_t)((K[i] % 64 + 15) / 16 * 16);
           st = encode_2d(&m[MAP_B_TAIL], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)K[i], (uint64_t)ldb[i],
-                         (uint32_t)(g.b_swz / 2), rows, g.b_swz);
+                         (uint32_t)(gb.b_swz / 2), rows, gb.b_swz);
           if (st != VB_OK) return st;
         }
       }
       // C box = one epilogue quarter's sub-box: c_cols x BY/4 rows
       st = encode_2d(&m[MAP_C], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)M[i], (uint64_t)ldc[i],
-                     (uint32_t)g.c_cols, (uint32_t)(s.BY / 4), g.c_swz);
+                     (uint32_t)g.c_cols, (uint32_t)(BYc / 4), g.c_swz);
       if (st != VB_OK) return st;
     }
   }
@@ -272,7 +276,7 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
     g.lda = lda[i];
     g.ldb = ldb[i];
     g.ldc = ldc[i];
-    g.row = p->tiling.row[i] | (s.BY << 8) | (s.BX << 16);
+    g.row = p->tiling.row[i] | ((s.BY / s.ctas) << 8) | (s.BX << 16);   // per-CTA rows
     g.kblocks = (int32_t)cdiv64(K[i], s.BK);
   }
   if (p->dt != VB_F32) {
@@ -324,16 +328,33 @@ extern "C" vb_status vb_plan_vbatched(int device, vb_dtype dt, int32_t batch, co
     p->batch = batch;
     p->table = t;
     p->policy = (int)policy;
-    p->tiling = tiling_engine(M, N, batch, *t, thr);
+    p->tiling = tiling_engine(M, N, batch, *t, thr, pairs_allowed(M, N, K, batch, elem_bytes(dt)));
     if (batch == 0) p->tiling.version_T = t->versions[0];
-    const std::vector<TileRec> tiles = enumerate_tiles(M, N, K, batch, p->tiling.row, *t);
-    if (tiles.size() > (size_t)INT32_MAX) {
+    const std::vector<TileRec> all = enumerate_tiles(M, N, K, batch, p->tiling.row, *t);
+    if (all.size() > (size_t)INT32_MAX) {
       delete p;
       return fail(VB_ERR_INVALID_ARG, "more than 2^31 tiles");
     }
-    Schedule sch = policy == VB_BATCH_THRESHOLD ? batch_threshold(tiles, p->tiling.version_T, thr, theta)
-                   : policy == VB_BATCH_BINARY  ? batch_binary(tiles, theta)
-                                                : batch_none(tiles);
+    // 2-SM pair tiles run in their own cluster kernel: batch them separately, pair blocks first.
+    std::vector<TileRec> tiles;
+    tiles.reserve(all.size());
+    for (const TileRec &r : all)
+      if (t->rows[p->tiling.row[r.gemm]].ctas == 2) tiles.push_back(r);
+    const size_t n_pair = tiles.size();
+    for (const TileRec &r : all)
+      if (t->rows[p->tiling.row[r.gemm]].ctas != 2) tiles.push_back(r);
+    Schedule sch;
+    sch.block_ptr.push_back(0);
+    for (int part = 0; part < 2; ++part) {
+      const std::vector<TileRec> sub(tiles.begin() + (part ? n_pair : 0), part ? tiles.end() : tiles.begin() + n_pair);
+      const Schedule sp = policy == VB_BATCH_THRESHOLD ? batch_threshold(sub, p->tiling.version_T, thr, theta)
+                          : policy == VB_BATCH_BINARY  ? batch_binary(sub, theta)
+                                                       : batch_none(sub);
+      const int32_t base = (int32_t)sch.slot_tile.size(), off = part ? (int32_t)n_pair : 0;
+      for (int32_t v : sp.slot_tile) sch.slot_tile.push_back(v + off);
+      for (size_t b = 1; b < sp.block_ptr.size(); ++b) sch.block_ptr.push_back(base + sp.block_ptr[b]);
+      if (part == 0) p->n_pair_blocks = (int)sch.block_ptr.size() - 1;
+    }
     st = finish_plan(p, M, N, K, lda, ldb, ldc, tiles, sch);
     if (st != VB_OK) {
       delete p;
@@ -395,12 +416,31 @@ extern "C" vb_status vb_plan_from_schedule(int device, vb_dtype dt, int32_t batc
       if (seen[(size_t)id]++) return fail(VB_ERR_INVALID_ARG, "slot %lld: tile covered twice", (long long)s);
       tiles[(size_t)s] = TileRec{g, tile_y[s], tile_x[s], K[g]};
     }
+    // 2-SM pair tiles need their own cluster kernel: blocks must not mix pair and 1-SM tiles,
+    // and the pair blocks must come first
+    int n_pair_blocks = 0;
+    bool single_seen = false;
+    for (int b = 0; b < n_blocks; ++b) {
+      int kind = -1;
+      for (int32_t k = block_ptr[b]; k < block_ptr[b + 1]; ++k) {
+        const int c = t->rows[gemm_row[tiles[(size_t)k].gemm]].ctas;
+        if (kind >= 0 && c != kind) return fail(VB_ERR_INVALID_ARG, "block %d mixes 2-SM and 1-SM tiles", b);
+        kind = c;
+      }
+      if (kind == 2) {
+        if (single_seen) return fail(VB_ERR_INVALID_ARG, "2-SM pair blocks must precede 1-SM blocks");
+        ++n_pair_blocks;
+      } else if (kind == 1) {
+        single_seen = true;
+      }
+    }
     vb_plan *p = new vb_plan();
     p->device = device;
     p->dt = dt;
     p->batch = batch;
     p->table = t;
     p->policy = -1;
+    p->n_pair_blocks = n_pair_blocks;
     p->tiling.row.assign(gemm_row, gemm_row + batch);
     p->tiling.version_T = version_T;
     Schedule sch;
@@ -468,8 +508,18 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
               alpha, beta};
     e = launch_f32(a, n_blocks, p->tiling.version_T, s);
   } else {
-    TcArgs a{p->d_block_ptr, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_blocks, g_trace};
-    e = launch_tc(a, std::min(n_blocks, p->sm_count), p->dt == VB_BF16, s);
+    // 2-SM pair tiles first (clusters of 2 over blocks [0, n_pair)), then the 1-SM tiles
+    const int n_pair = p->n_pair_blocks, n_single = n_blocks - n_pair;
+    e = cudaSuccess;
+    if (n_pair > 0) {
+      TcArgs a{p->d_block_ptr, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_pair, g_trace};
+      e = launch_tc(a, 2 * std::min(n_pair, p->sm_count / 2), p->dt == VB_BF16, true, s);
+    }
+    if (e == cudaSuccess && n_single > 0) {
+      TcArgs a{p->d_block_ptr + n_pair, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter + 2, n_single,
+               g_trace};
+      e = launch_tc(a, std::min(n_single, p->sm_count), p->dt == VB_BF16, false, s);
+    }
   }
   return e == cudaSuccess ? VB_OK : cuda_fail(e, "kernel launch");
 }
@@ -493,7 +543,10 @@ extern "C" vb_status vb_plan_info(vb_plan_t p, int64_t *n_tiles, int64_t *n_bloc
   if (version_T) *version_T = p->tiling.version_T;
   if (launches_per_exec) {
     const bool any = p->block_ptr.size() > 1;
-    *launches_per_exec = p->batch == 0 ? 0 : (p->dt == VB_F32 ? (any ? 1 : 0) : (any ? 2 : 1));  // prep + GEMM
+    const int nb = (int)p->block_ptr.size() - 1;
+    *launches_per_exec = p->batch == 0 ? 0
+                         : p->dt == VB_F32 ? (any ? 1 : 0)
+                                           : 1 + (p->n_pair_blocks > 0) + (nb - p->n_pair_blocks > 0);  // prep + GEMMs
   }
   return VB_OK;
 }

@@ -203,7 +203,10 @@ __device__ __forceinline__ void epi_row(uint8_t *cb, int row, int c_swz, int u0,
 }
 
 // --------------------------------------------------------------------------------- kernel
-template <int AB_FMT>
+// PAIR = the 2-SM variant (cluster of 2 CTAs, cta_group::2): every tile is a 256-row pair tile,
+// CTA r owns rows r*128.. of it and half of B; CTA 0 (the leader) schedules, issues the MMAs and
+// owns the barriers both CTAs' TMA loads and epilogues report to.
+template <int AB_FMT, bool PAIR>
 __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constant__ TcArgs p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -212,6 +215,21 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   Shared *sh = reinterpret_cast<Shared *>(cbuf + (size_t)kCSlots * kCSlotBytes);
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+  const uint32_t rank = PAIR ? ptx::cluster_ctarank() : 0u;
+  const bool leader = rank == 0;
+  // in a pair, consumers of the peer CTA release ring entries / accumulators on the leader
+  auto ring_release = [&](int e) {
+    if (!PAIR || leader)
+      ptx::mbar_arrive(&sh->rempty[e]);
+    else
+      ptx::mbar_arrive_remote(ptx::mapa(&sh->rempty[e], 0));
+  };
+  auto ring_wait = [&](int e, uint32_t ph) {
+    if (PAIR)
+      ptx::mbar_wait_cluster(&sh->rfull[e], ph);
+    else
+      ptx::mbar_wait(&sh->rfull[e], ph);
+  };
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < kSlots; ++i) {
@@ -220,7 +238,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     }
     for (int i = 0; i < kAcc; ++i) {
       ptx::mbar_init(&sh->tfull[i], 1);
-      ptx::mbar_init(&sh->tempty[i], kEpiWarps);
+      ptx::mbar_init(&sh->tempty[i], PAIR ? 2 * kEpiWarps : kEpiWarps);
     }
     for (int i = 0; i < kCSlots; ++i) {
       ptx::mbar_init(&sh->cfull[i], kCProducers);
@@ -228,14 +246,22 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     }
     for (int i = 0; i < kRing; ++i) {
       ptx::mbar_init(&sh->rfull[i], 1);
-      ptx::mbar_init(&sh->rempty[i], kRingConsumers);
+      ptx::mbar_init(&sh->rempty[i], PAIR ? 2 * kRingConsumers - 1 : kRingConsumers);   // peer has no MMA
     }
     sh->prod_kb = 0u;
     ptx::fence_mbar_init();
   }
-  if (warp == 1) ptx::tmem_alloc(&sh->tmem_base, kTmemCols);
+  if (warp == 1) {
+    if (PAIR)
+      ptx::tmem_alloc_pair(&sh->tmem_base, kTmemCols);
+    else
+      ptx::tmem_alloc(&sh->tmem_base, kTmemCols);
+  }
   ptx::tc_fence_before();
-  __syncthreads();
+  if (PAIR)
+    ptx::cluster_sync();   // both CTAs' barriers initialised before any remote arrive
+  else
+    __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = sh->tmem_base;
   const uint8_t *tmaps = reinterpret_cast<const uint8_t *>(p.tmaps);
@@ -245,7 +271,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   const long long t_start = clock64();
 #endif
 
-  if (warp == 0) {
+  if (warp == 0 && leader) {
     // ================================================================ scheduler (whole warp)
     // Tile t of this CTA goes to ring entry t % kRing with phase (t / kRing) & 1.
     // The lookahead is bounded in k-blocks (kKbAhead) rather than tiles, so CTAs working on
@@ -286,6 +312,14 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           ti.d = d;
           ti.alpha = al;
           ti.beta = be;
+          if (PAIR) {                                 // mirror the entry into the peer's ring
+            const uint32_t ra = ptx::mapa(&ti, 1);
+            const uint4 *src = reinterpret_cast<const uint4 *>(&ti);
+            ptx::st_cluster_v4(ra, src[0]);
+            ptx::st_cluster_v4(ra + 16, src[1]);
+            ptx::st_cluster_v4(ra + 32, src[2]);
+            ptx::mbar_arrive_remote(ptx::mapa(&sh->rfull[e], 1));
+          }
           ptx::mbar_arrive(&sh->rfull[e]);
         }
 #pragma unroll
@@ -299,8 +333,14 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const int e = (int)(t % kRing);
       ptx::mbar_wait(&sh->rempty[e], ((t / kRing) & 1u) ^ 1u);
       sh->ring[e].d.gemm = -1;
+      if (PAIR) {
+        asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(ptx::mapa(&sh->ring[e].d.gemm, 1)), "r"(-1) : "memory");
+        ptx::mbar_arrive_remote(ptx::mapa(&sh->rfull[e], 1));
+      }
       ptx::mbar_arrive(&sh->rfull[e]);
     }
+  } else if (warp == 0) {
+    // the peer CTA of a pair has no scheduler: the leader mirrors every ring entry into it
   } else if (warp >= 4 && warp < 8) {
     // ================================================================ A/B TMA producers
     // kProducers warps run the same deterministic page allocator over the same tile sequence
@@ -314,29 +354,40 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       uint32_t rph = 0, sph = 0, ophase = 0, kbg = 0;
       int32_t *slot_pages = sh->slot_pages[pid];
       for (;;) {
-        VB_TWAIT(T_PROD_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
+        VB_TWAIT(T_PROD_RFULL, ring_wait(re, rph));
         const TileInfo ti = sh->ring[re];
-        ptx::mbar_arrive(&sh->rempty[re]);
+        ring_release(re);
         advance(re, rph, kRing);
         if (ti.d.gemm < 0) break;
         if (ti.d.kblocks == 0) {
-          if (pid == 0) sh->prod_kb = sh->prod_kb + 1u;
+          if (pid == 0 && leader) sh->prod_kb = sh->prod_kb + 1u;
           continue;
         }
-        const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
-        const TcGeom geo = tc_geom(BY, BX);
+        // per-CTA geometry: a pair tile gives each CTA 128 rows of A and BX/2 columns of B
+        const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
+        const int BXc = PAIR ? BX / 2 : BX;
+        const TcGeom geo = tc_geom(BY, BXc);
         const uint8_t *maps = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128);
         // out-of-bounds box rows cost L2 bandwidth even though TMA zero-fills them: the last
         // row-tile uses the row-tail map, the last k-block the K-tail map, and B boxes that lie
         // entirely past N are not loaded (their MMA columns are discarded by the epilogue)
-        const int a_rows = min(BY, ti.d.M - ti.d.m0);
-        const bool a_tail = a_rows < BY;
+        // rows / B boxes this CTA loads, and (pair) what the peer loads, for the byte count
+        auto a_box_rows_of = [&](int r) {
+          const int rows = min(BY, ti.d.M - (ti.d.m0 + r * BY));
+          return rows <= 0 ? 0 : (rows < BY ? (rows + 7) / 8 * 8 : BY);
+        };
+        auto b_boxes_of = [&](int r) {
+          const int cols = ti.d.N - (ti.d.n0 + r * BXc);
+          return cols <= 0 ? 0 : min(geo.b_boxes, (cols + geo.b_swz / 2 - 1) / (geo.b_swz / 2));
+        };
+        const int row0 = ti.d.m0 + (int)rank * BY, col0 = ti.d.n0 + (int)rank * BXc;
+        const int a_box_rows = a_box_rows_of((int)rank);
+        const bool a_tail = a_box_rows != BY;
         const uint8_t *mapA = maps + (a_tail ? MAP_A_TAIL : MAP_A) * 128;
-        const int a_box_rows = a_tail ? (a_rows + 7) / 8 * 8 : BY;
-        const int b_boxes = min(geo.b_boxes, (ti.d.N - ti.d.n0 + geo.b_swz / 2 - 1) / (geo.b_swz / 2));
+        const int b_boxes = b_boxes_of((int)rank);
         const int ksteps_last = (ti.d.flags >> 8) & 7;
         const int a_pages = BY * kBK * 2 / kPageBytes;
-        const int need = a_pages + (BX * kBK * 2 + kPageBytes - 1) / kPageBytes;
+        const int need = a_pages + (BXc * kBK * 2 + kPageBytes - 1) / kPageBytes;
         for (int kb = 0; kb < ti.d.kblocks; ++kb, ++kbg) {
           int start = head, take = need;
           if (start + need > kPages) {          // never wrap a k-block around the ring end
@@ -367,38 +418,45 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           VB_T0();
           if (pid == 0) {
             sh->slot_page[slot] = start;
-            ptx::mbar_arrive_expect_tx(&sh->full[slot],
-                                       (uint32_t)(a_box_rows * kBK * 2 + b_boxes * b_rows * geo.b_swz));
+            if (leader) {                     // the leader's barrier counts both CTAs' bytes
+              uint32_t bytes = (uint32_t)(a_box_rows_of(0) * kBK * 2 + b_boxes_of(0) * b_rows * geo.b_swz);
+              if (PAIR) bytes += (uint32_t)(a_box_rows_of(1) * kBK * 2 + b_boxes_of(1) * b_rows * geo.b_swz);
+              ptx::mbar_arrive_expect_tx(&sh->full[slot], bytes);
+            }
           }
           // box 0 = A, boxes 1..b_boxes = B; box i goes to producer (i + kbg) % kProducers
           for (int i = (int)((pid - kbg) % kProducers + kProducers) % kProducers; i <= b_boxes; i += kProducers) {
-            if (i == 0)
-              ptx::tma_load_2d(sa, mapA, &sh->full[slot], kb * kBK, ti.d.m0);
+            if (i == 0 && a_box_rows == 0) continue;
+            uint8_t *dst = i == 0 ? sa : sb + (i - 1) * kBK * geo.b_swz;
+            const uint8_t *map = i == 0 ? mapA : mapB;
+            const int c0 = i == 0 ? kb * kBK : col0 + (i - 1) * (geo.b_swz / 2);
+            const int c1 = i == 0 ? row0 : kb * kBK;
+            if (PAIR)
+              ptx::tma_load_2d_pair(dst, map, &sh->full[slot], c0, c1);
             else
-              ptx::tma_load_2d(sb + (i - 1) * kBK * geo.b_swz, mapB, &sh->full[slot],
-                               ti.d.n0 + (i - 1) * (geo.b_swz / 2), kb * kBK);
+              ptx::tma_load_2d(dst, map, &sh->full[slot], c0, c1);
           }
           VB_TADD(T_PROD_ISSUE);
           advance(slot, sph, kSlots);
-          if (pid == 0) sh->prod_kb = sh->prod_kb + 1u;
+          if (pid == 0 && leader) sh->prod_kb = sh->prod_kb + 1u;
         }
       }
     }
   } else if (warp == 1) {
     // ================================================================ MMA issuer (+ TMEM owner)
-    if (lane == 0) {
+    if (lane == 0 && leader) {
       int re = 0, slot = 0, oldest = 0, free_units = kAccUnits, inflight = 0;
       uint32_t rph = 0, sph = 0, t = 0, ophase = 0;
       int32_t *acc_take = sh->acc_take;
       AccRing ring;
       for (;;) {
-        VB_TWAIT(T_MMA_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
+        VB_TWAIT(T_MMA_RFULL, ring_wait(re, rph));
         const TileInfo ti = sh->ring[re];
-        ptx::mbar_arrive(&sh->rempty[re]);
+        ring_release(re);
         advance(re, rph, kRing);
         if (ti.d.gemm < 0) break;
-        const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
-        const TcGeom geo = tc_geom(BY, BX);
+        const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);   // MMA shape (pair: M = 256)
+        const TcGeom geo = tc_geom(PAIR ? BY / 2 : BY, PAIR ? BX / 2 : BX);   // this CTA's B half
         const int e = (int)(t % kAcc);
         ++t;
 #ifdef VB_TRACE
@@ -423,7 +481,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const uint32_t d_tmem = tmem_base + (uint32_t)(start * kAccUnit);
         const uint32_t idesc = ptx::idesc_f16((uint32_t)AB_FMT, BY, BX);
         const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
-        const uint32_t a_bytes = (uint32_t)BY * kBK * 2;
+        const uint32_t a_bytes = (uint32_t)(PAIR ? BY / 2 : BY) * kBK * 2;
         for (int kb = 0; kb < ti.d.kblocks; ++kb) {
           VB_TWAIT(T_MMA_FULL, ptx::mbar_wait(&sh->full[slot], sph));
           ptx::tc_fence_after();
@@ -440,16 +498,25 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             // b_swz/2 elements 64*b_swz apart (LBO); K step of 16 rows = +16*b_swz bytes.
             const uint64_t bdesc = ptx::smem_desc(sb + kk * 16 * geo.b_swz, kBK * geo.b_swz, 8 * geo.b_swz, blayout);
 #ifndef VB_EXP_NOMMA
-            ptx::mma_f16_ss(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
+            if (PAIR)
+              ptx::mma_f16_ss_pair(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
+            else
+              ptx::mma_f16_ss(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
 #else
             (void)adesc; (void)bdesc; (void)idesc; (void)d_tmem;
 #endif
           }
-          ptx::mma_commit(&sh->empty[slot]);      // frees the k-block's pages when the MMAs retire
+          if (PAIR)
+            ptx::mma_commit_pair(&sh->empty[slot]);   // frees the k-block's pages in both CTAs
+          else
+            ptx::mma_commit(&sh->empty[slot]);      // frees the k-block's pages when the MMAs retire
           VB_TADD(T_MMA_ISSUE);
           advance(slot, sph, kSlots);
         }
-        ptx::mma_commit(&sh->tfull[e]);           // accumulator ready for the epilogue
+        if (PAIR)
+          ptx::mma_commit_pair(&sh->tfull[e]);
+        else
+          ptx::mma_commit(&sh->tfull[e]);           // accumulator ready for the epilogue
       }
     }
   } else if (warp == 2 || warp == 3) {
@@ -461,13 +528,14 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       uint32_t rph = 0, cph = 0;
       const uint64_t c_policy = ptx::policy_evict_first();
       for (;;) {
-        VB_TWAIT(T_CPROD_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
+        VB_TWAIT(T_CPROD_RFULL, ring_wait(re, rph));
         const TileInfo ti = sh->ring[re];
-        ptx::mbar_arrive(&sh->rempty[re]);
+        ring_release(re);
         advance(re, rph, kRing);
         if (ti.d.gemm < 0) break;
-        const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
+        const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
         const TcGeom geo = tc_geom(BY, BX);
+        const int row0 = ti.d.m0 + (int)rank * BY;
         const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C * 128;
         const bool load = ti.beta != 0.f;
         for (int ch = 0; ch < geo.c_chunks; ++ch) {
@@ -476,11 +544,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             // the C map's box is one epilogue quarter's sub-box (BY/4 rows); skip rows >= M
             const int rows_w = BY / 4;
             int nsub = 0;
-            for (int w = 2 * cid; w < 2 * cid + 2; ++w) nsub += (ti.d.m0 + w * rows_w < ti.d.M) ? 1 : 0;
+            for (int w = 2 * cid; w < 2 * cid + 2; ++w) nsub += (row0 + w * rows_w < ti.d.M) ? 1 : 0;
             ptx::mbar_arrive_expect_tx(&sh->cfull[cs], (uint32_t)(nsub * rows_w * geo.c_cols * 2));
             for (int w = 2 * cid; w < 2 * cid + nsub; ++w)
               ptx::tma_load_2d_hint(cbuf + (size_t)cs * kCSlotBytes + w * rows_w * geo.c_swz, mapC, &sh->cfull[cs],
-                                    ti.d.n0 + ch * geo.c_cols, ti.d.m0 + w * rows_w, c_policy);
+                                    ti.d.n0 + ch * geo.c_cols, row0 + w * rows_w, c_policy);
           } else {
             ptx::mbar_arrive(&sh->cfull[cs]);
           }
@@ -501,14 +569,15 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     uint32_t rph = 0, cph = 0, t = 0;
     AccRing acc_ring;
     for (;;) {
-      VB_TWAIT(T_EPI_RFULL, ptx::mbar_wait(&sh->rfull[re], rph));
+      VB_TWAIT(T_EPI_RFULL, ring_wait(re, rph));
       const TileInfo ti = sh->ring[re];
       __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&sh->rempty[re]);
+      if (lane == 0) ring_release(re);
       advance(re, rph, kRing);
       if (ti.d.gemm < 0) break;
-      const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);
+      const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
       const TcGeom geo = tc_geom(BY, BX);
+      const int row0 = ti.d.m0 + (int)rank * BY;     // this CTA's first row of the tile
       const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C * 128;
       const int e = (int)(t % kAcc);
       const uint32_t aph = (t / kAcc) & 1u;
@@ -521,7 +590,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const int r0 = q * rows_w;
       const int row = r0 + lane;
       const bool row_ok = lane < rows_w;
-      const bool live = ti.d.m0 + r0 < ti.d.M;          // any row of this quarter inside the GEMM
+      const bool live = row0 + r0 < ti.d.M;             // any row of this quarter inside the GEMM
       const bool has_acc = ti.d.kblocks > 0;
       const int hcols = geo.c_cols / 2;                  // this warp's columns of a chunk
       const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)acc_col + half * hcols;
@@ -541,7 +610,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       auto release_acc = [&]() {                       // accumulator drained: hand it back early
         ptx::tc_fence_before();
         __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&sh->tempty[e]);
+        if (lane == 0) {
+          if (!PAIR || leader)
+            ptx::mbar_arrive(&sh->tempty[e]);
+          else
+            ptx::mbar_arrive_remote(ptx::mapa(&sh->tempty[e], 0));
+        }
       };
       auto process = [&](int ch, const uint32_t *acc) {
         const int col0 = ti.d.n0 + ch * geo.c_cols;
@@ -578,7 +652,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 #else
             if (live) {
 #endif
-              ptx::tma_store_2d_hint(mapC, cb + r0 * geo.c_swz, col0, ti.d.m0 + r0, c_policy);
+              ptx::tma_store_2d_hint(mapC, cb + r0 * geo.c_swz, col0, row0 + r0, c_policy);
               ptx::bulk_commit();
             }
             if (pending >= 0) {
@@ -592,7 +666,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           // The chunk ends inside a 16-byte granule of the row (N % 8 != 0): a TMA store would
           // write the whole granule, past N into the caller's padding.  Store this warp's
           // columns from the thread's own row with exact per-element bounds instead.
-          const int grow = ti.d.m0 + row;
+          const int grow = row0 + row;
           if (row_ok && grow < ti.d.M) {
             const int c_lo = half * hcols;
             uint8_t *crow = static_cast<uint8_t *>(p.C[ti.d.gemm]) + ((size_t)grow * ti.d.ldc + col0) * 2;
@@ -642,9 +716,17 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 #endif
   __syncwarp();
   ptx::tc_fence_before();
-  __syncthreads();
+  if (PAIR)
+    ptx::cluster_sync();   // no peer MMA / remote arrive may still target this CTA
+  else
+    __syncthreads();
   ptx::tc_fence_after();
-  if (warp == 1) ptx::tmem_dealloc(tmem_base, kTmemCols);
+  if (warp == 1) {
+    if (PAIR)
+      ptx::tmem_dealloc_pair(tmem_base, kTmemCols);
+    else
+      ptx::tmem_dealloc(tmem_base, kTmemCols);
+  }
   // The last CTA to finish resets the work-list counter, so back-to-back launches of the
   // same bound plan need no reset kernel.  Every CTA fetched past n_blocks before getting here.
   if (threadIdx.x == 0) {
@@ -667,8 +749,8 @@ __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
                            const GemmParam *gemms, int batch, int32_t *counter) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i == 0) {
-    counter[0] = 0;
-    counter[1] = 0;
+    counter[0] = counter[1] = 0;   // pair kernel
+    counter[2] = counter[3] = 0;   // 1-SM kernel
   }
   if (i >= batch * kMapsPerGemm) return;
   const int g = i / kMapsPerGemm, w = i % kMapsPerGemm;
@@ -690,11 +772,13 @@ __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
 size_t tc_smem_bytes() { return tck::kSmemBytes; }
 
 cudaError_t tc_configure() {
-  cudaError_t e = cudaFuncSetAttribute(tck::vb_tc_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)tck::kSmemBytes);
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(tck::vb_tc_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              (int)tck::kSmemBytes);
+  cudaError_t e = cudaSuccess;
+  const int smem = (int)tck::kSmemBytes;
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  return e;
 }
 
 cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
@@ -704,13 +788,30 @@ cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
   return cudaGetLastError();
 }
 
-cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, cudaStream_t stream) {
+// grid = persistent CTAs; pair = launch as clusters of 2 (grid must be even)
+cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, cudaStream_t stream) {
   if (grid <= 0) return cudaSuccess;
-  if (bf16)
-    tck::vb_tc_kernel<1><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
-  else
-    tck::vb_tc_kernel<0><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
-  return cudaGetLastError();
+  if (!pair) {
+    if (bf16)
+      tck::vb_tc_kernel<1, false><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
+    else
+      tck::vb_tc_kernel<0, false><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
+    return cudaGetLastError();
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(tck::kThreads);
+  cfg.dynamicSmemBytes = tck::kSmemBytes;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return bf16 ? cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<1, true>, args)
+              : cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<0, true>, args);
 }
 
 }  // namespace vb

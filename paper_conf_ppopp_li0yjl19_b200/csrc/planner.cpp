@@ -26,14 +26,31 @@ int64_t tlp_eq1(const int32_t *M, const int32_t *N, int batch, const std::vector
   int64_t tiles = 0;
   for (int i = 0; i < batch; ++i) {
     const StrategyRow &s = t.rows[row[i]];
-    tiles += cdiv(M[i], s.BY) * cdiv(N[i], s.BX);
+    tiles += cdiv(M[i], s.BY) * cdiv(N[i], s.BX) * s.ctas;   // a pair tile occupies two CTAs
   }
   return tiles * (int64_t)T;
 }
 
+bool pairs_allowed(const int32_t *M, const int32_t *N, const int32_t *K, int batch, int elem_bytes) {
+  // exact in 128-bit integers (sums up to ~1e15 flops for 2^31 GEMMs of 2^20 x 2^20 x 2^31)
+  __int128 flops = 0, bytes = 0;
+  for (int i = 0; i < batch; ++i) {
+    flops += (__int128)2 * M[i] * N[i] * K[i];
+    if (M[i] > 0 && N[i] > 0)
+      bytes += (__int128)elem_bytes * ((int64_t)M[i] * K[i] + (int64_t)K[i] * N[i]) + (__int128)2 * elem_bytes * M[i] * N[i];
+  }
+  return bytes > 0 && flops >= (__int128)128 * bytes;
+}
+
 TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const TableDef &t,
-                        int64_t threshold) {
-  const std::vector<int> order = priority_order(t);
+                        int64_t threshold, bool allow_pairs) {
+  std::vector<int> order = priority_order(t);
+  if (!allow_pairs) {   // C-7b: the 1-SM version only
+    std::vector<int> o1;
+    for (int r : order)
+      if (t.rows[r].ctas == 1) o1.push_back(r);
+    order = o1;
+  }
   // Step 1 (P249): per-GEMM queue of strategies with BY <= M and BX <= N (C-1, with the
   // table's MMA floor C-1b); if none
   // fits, the smallest strategy alone (C-4).  A queue is a [head, end) window of `order`

@@ -30,13 +30,17 @@ struct Schedule {                  // the five auxiliary arrays of Fig. 6 (P282)
   std::vector<int32_t> slot_tile;  // slot -> tile index (enumeration order)
 };
 
-// Eq. 1 (P220) with ceil tile counts (reading C-5).
+// Eq. 1 (P220) with ceil tile counts (reading C-5); a 2-SM pair tile counts twice.
 int64_t tlp_eq1(const int32_t *M, const int32_t *N, int batch, const std::vector<int> &row,
                 const TableDef &t, int T);
 
 // §4.2.3 steps 1-3 and the two exceptions (P249-253; readings C-1..C-8).
 TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const TableDef &t,
-                        int64_t threshold);
+                        int64_t threshold, bool pairs_allowed = true);
+
+// Reading C-7b: offer the 2-SM pair strategies only to batches with arithmetic intensity
+// 2*sum(MNK) / sum(es*(MK+KN) + 2*es*MN) >= 128 flop/byte.
+bool pairs_allowed(const int32_t *M, const int32_t *N, const int32_t *K, int batch, int elem_bytes);
 
 // GEMM-major, row-major (y, x) tiles (P133-135, P157, P284; C-11, C-13).
 std::vector<TileRec> enumerate_tiles(const int32_t *M, const int32_t *N, const int32_t *K,

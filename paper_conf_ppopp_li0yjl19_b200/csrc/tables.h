@@ -10,9 +10,10 @@ struct StrategyRow {
   int BY;   // C-tile rows    (along M)
   int BX;   // C-tile columns (along N)
   int BK;   // K step of one main-loop iteration
+  int ctas;   // CTAs (SMs) that execute one tile: 2 = tcgen05 cta_group::2 pair tile
 };
 
-constexpr int kMaxRows = 8;
+constexpr int kMaxRows = 11;
 constexpr int kMaxVersions = 2;
 
 struct TableDef {
@@ -35,8 +36,8 @@ struct TableDef {
 // PAPER.md Table 2 (P204-214): small 16x16, medium 32x32, large 64x64, tall 128x64,
 // wide 64x128, huge 128x128; BK = 8 (P243); 256- and 128-thread versions (P181, P198).
 #define VB_TABLE2_ROWS                                                              \
-  {{"small", 16, 16, 8}, {"medium", 32, 32, 8}, {"large", 64, 64, 8},               \
-   {"tall", 128, 64, 8}, {"wide", 64, 128, 8}, {"huge", 128, 128, 8}}
+  {{"small", 16, 16, 8, 1}, {"medium", 32, 32, 8, 1}, {"large", 64, 64, 8, 1},      \
+   {"tall", 128, 64, 8, 1}, {"wide", 64, 128, 8, 1}, {"huge", 128, 128, 8, 1}}
 
 // V100 profile: the paper's constants (P255, P290).
 constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 128}, 65536, 256, 0, 0};
@@ -46,12 +47,16 @@ constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 1
 constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 2, {256, 128}, 131072, 256, 0, 0};
 
 // B200 tcgen05 profile (bf16/fp16): C tiles for tcgen05.mma with M in {64,128}; BK = 64 =
-// one 128-byte swizzled row of bf16; one kernel version with 256 threads (8 warps).  Besides
-// the paper's square/tall/wide family it has the skinny shapes 128x32 and 64x256 that
-// variable-size batches need once short GEMMs may take the 64-row MMA (min_BY = 64).
-constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 8,
-                                   {{"s", 64, 32, 64}, {"n", 128, 32, 64}, {"m", 64, 64, 64}, {"t", 128, 64, 64},
-                                    {"w", 64, 128, 64}, {"l", 128, 128, 64}, {"x", 64, 256, 64}, {"h", 128, 256, 64}},
+// one 128-byte swizzled row of bf16; 256 threads per tile in Eq. 1.  Besides the paper's
+// square/tall/wide family it has the skinny shapes 128x32 and 64x256 that variable-size
+// batches need once short GEMMs may take the 64-row MMA (min_BY = 64), and three 2-SM pair
+// tiles (cta_group::2, M = 256: each SM holds 128 rows of A and half of B, so a 256x256 pair
+// moves 33% fewer bytes per SM per k-block than 128x256) — the B200 "second version" of P198.
+constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 11,
+                                   {{"s", 64, 32, 64, 1}, {"n", 128, 32, 64, 1}, {"m", 64, 64, 64, 1},
+                                    {"t", 128, 64, 64, 1}, {"w", 64, 128, 64, 1}, {"l", 128, 128, 64, 1},
+                                    {"x", 64, 256, 64, 1}, {"h", 128, 256, 64, 1},
+                                    {"T2", 256, 64, 64, 2}, {"L2", 256, 128, 64, 2}, {"H2", 256, 256, 64, 2}},
                                    1, {256, 0}, 4 * 148 * 256, 512, 64, 32};
 
 #undef VB_TABLE2_ROWS

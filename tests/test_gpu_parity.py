@@ -111,6 +111,8 @@ def test_tc_edge_shapes(dtype, policy):
 def _forced_rows_plan(db, rows, table, table_id):
     """Device plan with the given strategy row per GEMM, one tile per block (plan_from_schedule)."""
     tiles = pr.enumerate_tiles(db.M, db.N, db.K, rows, table)
+    pair = [table.rows[rows[t.gemm]].ctas == 2 for t in tiles]     # 2-SM pair blocks first
+    tiles = [t for t, q in zip(tiles, pair) if q] + [t for t, q in zip(tiles, pair) if not q]
     return vb.plan_from_schedule(db.M, db.N, db.K, db.lda, db.ldb, db.ldc, rows, table.versions[0],
                                  list(range(len(tiles) + 1)), [t.gemm for t in tiles], [t.y for t in tiles],
                                  [t.x for t in tiles], dtype=db.dtype, device=0, table_id=table_id)
@@ -264,3 +266,28 @@ def test_rebind_alternating_buffers_never_uses_stale_descriptors(dtype):
         db.run(plan)                   # bind (patch maps) + GEMM kernel
         torch.cuda.synchronize()
         check_batch(db, range(len(M)), seeds[i], "random")
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f16"])
+def test_pair_tiles_selected_for_compute_bound_batch(dtype):
+    # arithmetic intensity ~200 flop/B >= 128: the tiler offers the 2-SM pair strategies (C-7b);
+    # shapes include row/column/K tails and a GEMM too short for a pair tile
+    M = np.array([512, 300, 777, 1024, 100, 256]); N = np.array([512, 260, 640, 1000, 96, 512])
+    K = np.array([2048, 1500, 1900, 4096, 3000, 2000])
+    db = DeviceBatch(M, N, K, dtype)
+    db.C.fill_(float("nan"))
+    db.fill(SEED)
+    plan = db.plan(tlp_threshold=1)        # small batch: let the tiler reach the largest tiles
+    ids = plan.export()["gemm_strategy"]
+    assert (ids >= 8).sum() >= 4 and plan.info()["launches_per_exec"] == 3, (ids, plan.info())
+    db.run(plan)
+    torch.cuda.synchronize()
+    check_batch(db, range(len(M)), SEED, "random")
+    _padding_untouched(db)
+
+
+def test_memory_bound_batch_keeps_one_sm_tiles():
+    M, N, K = vbinputs.config_sizes("C5")
+    assert not pr.pairs_allowed(M, N, K)
+    M, N, K = vbinputs.config_sizes("C4")
+    assert pr.pairs_allowed(M, N, K)
