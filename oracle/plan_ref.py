@@ -52,8 +52,9 @@ V100 = Table("v100_table2", (
     versions=(256, 128), tlp_threshold=65536, theta=256)
 
 # B200 FFMA (fp32) profile: the Table 2 shapes and sub-tiles are an FFMA design and are
-# kept; the platform constants are re-set for 148 SMs (reading C-22).
-B200_F32 = Table("b200_ffma", V100.rows, versions=(256, 128), tlp_threshold=131072, theta=256)
+# kept; the platform constants are re-set for 148 SMs and only the 256-thread version is
+# offered (calibrated on B200, reading C-22).
+B200_F32 = Table("b200_ffma", V100.rows, versions=(256,), tlp_threshold=131072, theta=256)
 
 # B200 tcgen05 (bf16/fp16) profile: C-tile shapes sized for tcgen05.mma
 # (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16), plus the skinny shapes

@@ -25,6 +25,7 @@ cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
                            const GemmParam *gemms, int batch, int32_t *counter, cudaStream_t stream);
 cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, cudaStream_t stream);
 cudaError_t tc_configure();
+cudaError_t f32_configure();
 size_t tc_smem_bytes();
 cudaError_t launch_fill(int dt, int batch, const int32_t *rows, const int32_t *cols, const int32_t *ld,
                         void *const *ptrs, const int64_t *gemm_id, uint64_t seed, int operand, int64_t total_elems,
@@ -204,6 +205,10 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   p->d_tiles = tc ? reinterpret_cast<TileDesc *>(base + o_td) : nullptr;
   p->d_tmaps = tc ? base + o_tm : nullptr;
 
+  if (!tc) {
+    e = f32_configure();
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(f32 kernel smem)");
+  }
   std::vector<uint8_t> host(p->ws_bytes, 0);
   memcpy(host.data() + o_bp, p->block_ptr.data(), p->block_ptr.size() * sizeof(int32_t));
   if (!p->slots.empty()) memcpy(host.data() + o_sl, p->slots.data(), p->slots.size() * sizeof(TileSlot));

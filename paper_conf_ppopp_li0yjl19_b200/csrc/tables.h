@@ -43,8 +43,10 @@ struct TableDef {
 constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 128}, 65536, 256, 0, 0};
 
 // B200 FFMA profile (fp32): Table 2 shapes/sub-tiles (an FFMA design that still holds on
-// sm_100a), threshold re-set for 148 SMs (reading C-22, calibration is NEXT-1).
-constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 2, {256, 128}, 131072, 256, 0, 0};
+// sm_100a), threshold re-set for 148 SMs (reading C-22).  Calibrated on B200: the 128-thread
+// version (16x8 sub-tiles, 255 registers, 8 warps per SM) is 13% slower than the 256-thread
+// version at two CTAs per SM on C2, so this profile offers the 256-thread version only.
+constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 1, {256, 0}, 131072, 256, 0, 0};
 
 // B200 tcgen05 profile (bf16/fp16): C tiles for tcgen05.mma with M in {64,128}; BK = 64 =
 // one 128-byte swizzled row of bf16; 256 threads per tile in Eq. 1.  Besides the paper's
