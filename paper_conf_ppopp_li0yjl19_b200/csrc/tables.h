@@ -26,9 +26,11 @@ struct TableDef {
   int64_t tlp_threshold;        // P253 / P290 (platform constant)
   int theta;                    // P259 / P290 (platform constant)
   // Availability floor (reading C-1b): a strategy is available for a GEMM when
-  // BY <= max(M, min_BY) and BX <= max(N, min_BX).  0 for the paper's tables (P249 exactly);
-  // for tcgen05 the MMA cannot be shorter than 64 rows, so min_BY = 64 (and min_BX = 32,
-  // the narrowest strategy): a 20-row GEMM occupies a 64-row MMA whichever tile it gets.
+  // BY <= max(M, min_BY) and BX <= max(N, min_BX).  0 for the paper's tables (P249 exactly).
+  // tcgen05 table: min_BY = 128 because an M = 64 MMA takes as many cycles as M = 128 (the
+  // pacing floor max(M,128)*N/256) and the rows past M are neither loaded (row-tail map) nor
+  // stored; min_BX = 64 because 64-column boxes use the 128-byte swizzle while narrower ones
+  // move at half the TMA rate (measured, tools/tma_bench.cu).
   int min_BY;
   int min_BX;
 };
@@ -59,7 +61,7 @@ constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 11,
                                     {"t", 128, 64, 64, 1}, {"w", 64, 128, 64, 1}, {"l", 128, 128, 64, 1},
                                     {"x", 64, 256, 64, 1}, {"h", 128, 256, 64, 1},
                                     {"T2", 256, 64, 64, 2}, {"L2", 256, 128, 64, 2}, {"H2", 256, 256, 64, 2}},
-                                   1, {256, 0}, 4 * 148 * 256, 512, 64, 32};
+                                   1, {256, 0}, 4 * 148 * 256, 512, 128, 64};
 
 #undef VB_TABLE2_ROWS
 
