@@ -252,6 +252,11 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
       st = encode_2d(&m[MAP_C], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)M[i], (uint64_t)ldc[i],
                      (uint32_t)g.c_cols, (uint32_t)(BYc / 4), g.c_swz);
       if (st != VB_OK) return st;
+      if (N[i] >= 8) {
+        st = encode_2d(&m[MAP_C_ST], p->dt, p->d_ws, (uint64_t)(N[i] & ~7), (uint64_t)M[i], (uint64_t)ldc[i],
+                       (uint32_t)g.c_cols, (uint32_t)(BYc / 4), g.c_swz);
+        if (st != VB_OK) return st;
+      }
     }
   }
   e = cudaMemcpy(p->d_ws, host.data(), p->ws_bytes, cudaMemcpyHostToDevice);
@@ -300,7 +305,8 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
       d.N = g.N;
       d.ldc = g.ldc;
       d.geo = (uint16_t)((s.BY / 16) | ((s.BX / 16) << 8));
-      // last C chunk of this tile ends inside a 16-byte granule of the row -> direct stores
+      // last C chunk of this tile ends inside a 16-byte granule of the row -> its partial
+      // granule is stored directly
       const int last_chunk_end = d.n0 + s.BX;
       d.flags = (uint16_t)(((g.N & 7) != 0 && last_chunk_end > g.N && d.n0 < g.N) ? 1 : 0);
       if (g.K % 64) d.flags |= (uint16_t)(((g.K % 64 + 15) / 16) << 8);   // MMA K-steps of the last k-block

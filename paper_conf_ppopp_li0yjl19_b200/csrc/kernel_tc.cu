@@ -93,7 +93,8 @@ constexpr size_t kSmemBytes = 1024 /*align slack*/ + (size_t)kPages * kPageBytes
 enum TraceSlot {
   T_SCHED_REMPTY, T_SCHED_BUDGET, T_PROD_RFULL, T_PROD_EMPTY, T_MMA_RFULL, T_MMA_TEMPTY, T_MMA_FULL,
   T_CPROD_RFULL, T_CPROD_CEMPTY, T_EPI_RFULL, T_EPI_TFULL, T_EPI_CFULL, T_EPI_STORE, T_EPI_TMEM, T_EPI_MATH,
-  T_TOTAL, T_TILES, T_PROD_ISSUE, T_MMA_ISSUE, T_EPI_FENCEBAR, T_EPI_STISSUE, T_EPI_LOOP, kTraceSlots
+  T_TOTAL, T_TILES, T_PROD_ISSUE, T_MMA_ISSUE, T_EPI_FENCEBAR, T_EPI_STISSUE, T_EPI_LOOP,
+  T_EPI_TLOAD, T_EPI_REL, T_EPI_PROC, T_EPI_HEAD, kTraceSlots
 };
 #ifdef VB_TRACE
 #define VB_T0() const long long _vbt0 = clock64()
@@ -304,6 +305,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             ptx::prefetch_tmap(maps + MAP_B * 128);
           }
           ptx::prefetch_tmap(maps + MAP_C * 128);
+          if (d.N >= 8) ptx::prefetch_tmap(maps + MAP_C_ST * 128);
           const float al = p.alpha[d.gemm], be = p.beta[d.gemm];
           const uint32_t tt = t + lane;
           const int e = (int)(tt % kRing);
@@ -570,6 +572,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     AccRing acc_ring;
     for (;;) {
       VB_TWAIT(T_EPI_RFULL, ring_wait(re, rph));
+#ifdef VB_TRACE
+      const long long _head_t0 = clock64();
+#endif
       const TileInfo ti = sh->ring[re];
       __syncwarp();
       if (lane == 0) ring_release(re);
@@ -578,7 +583,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
       const TcGeom geo = tc_geom(BY, BX);
       const int row0 = ti.d.m0 + (int)rank * BY;     // this CTA's first row of the tile
-      const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C * 128;
+      const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C_ST * 128;
+      const int n8 = ti.d.N & ~7;                       // the store map's width
       const int e = (int)(t % kAcc);
       const uint32_t aph = (t / kAcc) & 1u;
       ++t;
@@ -594,6 +600,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const bool has_acc = ti.d.kblocks > 0;
       const int hcols = geo.c_cols / 2;                  // this warp's columns of a chunk
       const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)acc_col + half * hcols;
+#ifdef VB_TRACE
+      tr[T_EPI_HEAD] += clock64() - _head_t0;
+#endif
       VB_TWAIT(T_EPI_TFULL, ptx::mbar_wait(&sh->tfull[e], aph));
       ptx::tc_fence_after();
 #ifdef VB_TRACE
@@ -619,12 +628,6 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       };
       auto process = [&](int ch, const uint32_t *acc) {
         const int col0 = ti.d.n0 + ch * geo.c_cols;
-        const bool direct = (ti.d.flags & 1) && (col0 + geo.c_cols > ti.d.N);
-        if (storer && lane == 0 && direct && pending >= 0) {   // keep at most one store pending
-          ptx::bulk_wait_read0();
-          ptx::mbar_arrive(&sh->cempty[pending]);
-          pending = -1;
-        }
         VB_TWAIT(T_EPI_CFULL, ptx::mbar_wait(&sh->cfull[cs], cph));
         uint8_t *cb = cbuf + (size_t)cs * kCSlotBytes;
         {
@@ -641,50 +644,41 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           }
           VB_TADD(T_EPI_MATH);
         }
-        if (!direct) {
-          // TMA store of the quarter's sub-box; rows >= M and whole 16-byte granules >= N are
-          // clipped by the TMA unit.
-          VB_TWAIT(T_EPI_FENCEBAR, ptx::fence_proxy_async_smem(); ptx::named_bar_sync(1 + q, 64));
-          VB_T0();
-          if (storer && lane == 0) {
-#ifdef VB_EXP_NOSTORE
-            if (false) {
-#else
-            if (live) {
-#endif
-              ptx::tma_store_2d_hint(mapC, cb + r0 * geo.c_swz, col0, row0 + r0, c_policy);
-              ptx::bulk_commit();
-            }
-            if (pending >= 0) {
-              VB_TWAIT(T_EPI_STORE, ptx::bulk_wait_read1());   // the previous store has read its slot
-              ptx::mbar_arrive(&sh->cempty[pending]);
-            }
-            pending = cs;
-          }
-          VB_TADD(T_EPI_STISSUE);
-        } else {
-          // The chunk ends inside a 16-byte granule of the row (N % 8 != 0): a TMA store would
-          // write the whole granule, past N into the caller's padding.  Store this warp's
-          // columns from the thread's own row with exact per-element bounds instead.
+        if ((ti.d.flags & 1) && col0 + geo.c_cols > ti.d.N) {
+          // The chunk ends inside the row's last, partial 16-byte granule (N % 8 != 0): the TMA
+          // store below stops at N & ~7, and the thread that computed the granule stores its
+          // N % 8 elements itself.
+          const int g0 = n8 - col0;                      // granule's first column in the chunk
           const int grow = row0 + row;
-          if (row_ok && grow < ti.d.M) {
-            const int c_lo = half * hcols;
-            uint8_t *crow = static_cast<uint8_t *>(p.C[ti.d.gemm]) + ((size_t)grow * ti.d.ldc + col0) * 2;
-            const int ncol = min(ti.d.N - col0, c_lo + hcols);
-            for (int c = c_lo; c < ncol; c += 8) {
-              const uint4 w =
-                  *reinterpret_cast<const uint4 *>(cb + ptx::swz((uint32_t)(row * geo.c_swz + c * 2), geo.c_swz));
-              if (c + 8 <= ncol) {
-                *reinterpret_cast<uint4 *>(crow + c * 2) = w;
-              } else {
-                const uint16_t *h = reinterpret_cast<const uint16_t *>(&w);
-                for (int e = 0; e < ncol - c; ++e) reinterpret_cast<uint16_t *>(crow + c * 2)[e] = h[e];
-              }
-            }
+          if (g0 >= half * hcols && g0 < (half + 1) * hcols && row_ok && grow < ti.d.M) {
+            const uint4 w = *reinterpret_cast<const uint4 *>(cb + ptx::swz((uint32_t)(row * geo.c_swz + g0 * 2), geo.c_swz));
+            const uint16_t *h = reinterpret_cast<const uint16_t *>(&w);
+            uint16_t *crow = reinterpret_cast<uint16_t *>(static_cast<uint8_t *>(p.C[ti.d.gemm]) +
+                                                          ((size_t)grow * ti.d.ldc + n8) * 2);
+            for (int j = 0; j < (ti.d.N & 7); ++j) crow[j] = h[j];
           }
-          ptx::named_bar_sync(1 + q, 64);
-          if (storer && lane == 0) ptx::mbar_arrive(&sh->cempty[cs]);
         }
+        // TMA store of the quarter's sub-box; rows >= M and columns >= N & ~7 are clipped by the
+        // TMA unit.  Every chunk commits one bulk group (possibly empty), so "all but the newest
+        // group have read their smem" always covers the previous chunk's slot.
+        VB_TWAIT(T_EPI_FENCEBAR, ptx::fence_proxy_async_smem(); ptx::named_bar_sync(1 + q, 64));
+        VB_T0();
+        if (storer && lane == 0) {
+#ifdef VB_EXP_NOSTORE
+          if (false) {
+#else
+          if (live && col0 < n8) {
+#endif
+            ptx::tma_store_2d_hint(mapC, cb + r0 * geo.c_swz, col0, row0 + r0, c_policy);
+          }
+          ptx::bulk_commit();
+          if (pending >= 0) {
+            VB_TWAIT(T_EPI_STORE, ptx::bulk_wait_read1());   // the previous store has read its slot
+            ptx::mbar_arrive(&sh->cempty[pending]);
+          }
+          pending = cs;
+        }
+        VB_TADD(T_EPI_STISSUE);
         advance(cs, cph, kCSlots);
       };
 
@@ -696,11 +690,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       }
       for (int ch = 0; ch < nch; ++ch) {
         if (has_acc) {
-          tload(ch, a0);
+          VB_TWAIT(T_EPI_TLOAD, tload(ch, a0));
           VB_TWAIT(T_EPI_TMEM, ptx::tmem_ld_wait());
         }
-        if (ch + 1 == nch) release_acc();
-        process(ch, a0);
+        if (ch + 1 == nch) VB_TWAIT(T_EPI_REL, release_acc());
+        VB_TWAIT(T_EPI_PROC, process(ch, a0));
       }
 #ifdef VB_TRACE
       tr[T_EPI_LOOP] += clock64() - _tile_t0;
@@ -757,9 +751,10 @@ __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
   const GemmParam gp = gemms[g];
   if (gp.M <= 0 || gp.N <= 0) return;
   const int BY = (gp.row >> 8) & 0xFF;
-  if (w != MAP_C && gp.K <= 0) return;
+  if (w != MAP_C && w != MAP_C_ST && gp.K <= 0) return;
   if (w == MAP_A_TAIL && gp.M % BY == 0) return;        // map not encoded
   if (w == MAP_B_TAIL && gp.K % 64 == 0) return;
+  if (w == MAP_C_ST && gp.N < 8) return;
   const void *ptr = (w == MAP_A || w == MAP_A_TAIL) ? A[g]
                     : (w == MAP_B || w == MAP_B_TAIL) ? B[g]
                                                       : static_cast<const void *>(C[g]);

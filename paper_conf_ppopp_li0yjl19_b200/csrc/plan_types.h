@@ -46,14 +46,16 @@ struct alignas(16) TileDesc {
   int32_t M, N;      // GEMM extents
   int32_t ldc;       // elements
   uint16_t geo;      // (BY / 16) | (BX / 16) << 8
-  uint16_t flags;    // bit 0: the tile's last C chunk ends inside a 16-byte granule (N % 8 != 0)
+  uint16_t flags;    // bit 0: the tile's last C chunk ends inside a 16-byte granule (N % 8 != 0):
+                     //        its columns [N & ~7, N) are stored directly, not by TMA
                      // bits 8-10: K=16 MMA steps of the last k-block (1..4), 0 = 4
 };
-// Tensor maps per GEMM (128 bytes each): A, A row-tail, B, B K-tail, C.  The tail maps have
-// boxes that stop at the matrix edge, because out-of-bounds box rows are zero-filled but still
-// cost L2 request bandwidth.
-constexpr int kMapsPerGemm = 5;
-enum MapIndex { MAP_A = 0, MAP_A_TAIL = 1, MAP_B = 2, MAP_B_TAIL = 3, MAP_C = 4 };
+// Tensor maps per GEMM (128 bytes each): A, A row-tail, B, B K-tail, C (loads), C store.  The
+// tail maps have boxes that stop at the matrix edge, because out-of-bounds box rows are
+// zero-filled but still cost L2 request bandwidth.  The C store map is N & ~7 columns wide:
+// a TMA store writes whole 16-byte granules, so clipping at N itself would write past N.
+constexpr int kMapsPerGemm = 6;
+enum MapIndex { MAP_A = 0, MAP_A_TAIL = 1, MAP_B = 2, MAP_B_TAIL = 3, MAP_C = 4, MAP_C_ST = 5 };
 static_assert(sizeof(TileDesc) == 32, "TileDesc must stay 32 bytes");
 
 struct TcArgs {

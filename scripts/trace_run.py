@@ -18,7 +18,8 @@ from paper_conf_ppopp_li0yjl19_b200.batch import DeviceBatch  # noqa: E402
 
 NAMES = ["sched_rempty", "sched_budget", "prod_rfull", "prod_empty", "mma_rfull", "mma_tempty", "mma_full",
          "cprod_rfull", "cprod_cempty", "epi_rfull", "epi_tfull", "epi_cfull", "epi_store", "epi_tmem", "epi_math",
-         "total", "tiles", "prod_issue", "mma_issue", "epi_fencebar", "epi_stissue", "epi_loop"]
+         "total", "tiles", "prod_issue", "mma_issue", "epi_fencebar", "epi_stissue", "epi_loop",
+         "epi_tload", "epi_rel", "epi_proc", "epi_head"]
 WARPS = {"sched": 1, "prod": 1, "mma": 1, "cprod": 1, "epi": 8, "cprod": 2, "prod": 4}
 
 ap = argparse.ArgumentParser()
