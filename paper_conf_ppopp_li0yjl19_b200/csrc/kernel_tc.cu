@@ -210,7 +210,9 @@ __device__ __forceinline__ void epi_row(uint8_t *cb, int row, int c_swz, int u0,
 template <int AB_FMT, bool PAIR>
 __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constant__ TcArgs p) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-byte aligned (SW128 atoms); offsetting smem_raw itself keeps the shared address space
+  // visible to the compiler, so C-slot and barrier accesses compile to LDS/STS, not generic LD/ST.
+  uint8_t *smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t *pages = smem;
   uint8_t *cbuf = smem + (size_t)kPages * kPageBytes;
   Shared *sh = reinterpret_cast<Shared *>(cbuf + (size_t)kCSlots * kCSlotBytes);
@@ -380,7 +382,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         };
         auto b_boxes_of = [&](int r) {
           const int cols = ti.d.N - (ti.d.n0 + r * BXc);
-          return cols <= 0 ? 0 : min(geo.b_boxes, (cols + geo.b_swz / 2 - 1) / (geo.b_swz / 2));
+          const int bw = geo.b_swz / 2;                  // a power of two: shift, not divide
+          return cols <= 0 ? 0 : min(geo.b_boxes, (cols + bw - 1) >> (__ffs(bw) - 1));
         };
         const int row0 = ti.d.m0 + (int)rank * BY, col0 = ti.d.n0 + (int)rank * BXc;
         const int a_box_rows = a_box_rows_of((int)rank);

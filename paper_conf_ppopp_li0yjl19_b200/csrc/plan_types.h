@@ -85,10 +85,10 @@ __host__ __device__ inline TcGeom tc_geom(int BY, int BX) {
   g.BY = BY;
   g.BX = BX;
   g.b_swz = BX >= 64 ? 128 : BX * 2;
-  g.b_boxes = BX / (g.b_swz / 2);
+  g.b_boxes = BX >= 64 ? BX >> 6 : 1;      // BX / (b_swz / 2), without an integer division
   g.c_cols = BX >= 64 ? 64 : BX;
   g.c_swz = g.c_cols * 2;
-  g.c_chunks = BX / g.c_cols;
+  g.c_chunks = BX >= 64 ? BX >> 6 : 1;     // BX / c_cols
   return g;
 }
 
