@@ -52,6 +52,18 @@ constexpr int kPageBytes = 8192;
 #ifndef VB_KBAHEAD
 #define VB_KBAHEAD 24
 #endif
+// L2 evict-first hints on the C_old loads / C stores.  Measured off by default: with the load
+// hint, C5 read 1.3x its compulsory DRAM bytes (a 500^3 batch: C_old fetched ~1.6x) and ran
+// 6% slower; without it DRAM reads are within 1-2% of the compulsory bytes.
+#ifndef VB_CLOAD_HINT
+#define VB_CLOAD_HINT 0
+#endif
+#ifndef VB_CSTORE_HINT
+#define VB_CSTORE_HINT 0
+#endif
+#ifndef VB_AB_HINT
+#define VB_AB_HINT 0      // experiment: A/B loads marked L2 evict-last
+#endif
 constexpr int kPages = VB_PAGES;           // 144 KB of A/B staging (default)
 constexpr int kSlots = 16;                 // k-blocks in flight (bounded by pages anyway)
 constexpr int kCSlots = VB_CSLOTS;
@@ -353,6 +365,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     // arms the full barrier (arrive + expect_tx of the k-block's total bytes), publishes the
     // k-block's page, and reports progress to the scheduler.
     const int pid = warp - 4;
+    const uint64_t ab_policy = ptx::policy_evict_last();
+    (void)ab_policy;
     if (lane == 0 && pid < kProducers) {
       int re = 0, slot = 0, head = 0, oldest = 0, inflight = 0, free_pages = kPages;
       uint32_t rph = 0, sph = 0, ophase = 0, kbg = 0;
@@ -439,7 +453,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             if (PAIR)
               ptx::tma_load_2d_pair(dst, map, &sh->full[slot], c0, c1);
             else
+#if VB_AB_HINT
+              ptx::tma_load_2d_hint(dst, map, &sh->full[slot], c0, c1, ab_policy);
+#else
               ptx::tma_load_2d(dst, map, &sh->full[slot], c0, c1);
+#endif
           }
           VB_TADD(T_PROD_ISSUE);
           advance(slot, sph, kSlots);
@@ -532,6 +550,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       int re = 0, cs = 0;
       uint32_t rph = 0, cph = 0;
       const uint64_t c_policy = ptx::policy_evict_first();
+      (void)c_policy;
       for (;;) {
         VB_TWAIT(T_CPROD_RFULL, ring_wait(re, rph));
         const TileInfo ti = sh->ring[re];
@@ -552,8 +571,13 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             for (int w = 2 * cid; w < 2 * cid + 2; ++w) nsub += (row0 + w * rows_w < ti.d.M) ? 1 : 0;
             ptx::mbar_arrive_expect_tx(&sh->cfull[cs], (uint32_t)(nsub * rows_w * geo.c_cols * 2));
             for (int w = 2 * cid; w < 2 * cid + nsub; ++w)
+#if VB_CLOAD_HINT
               ptx::tma_load_2d_hint(cbuf + (size_t)cs * kCSlotBytes + w * rows_w * geo.c_swz, mapC, &sh->cfull[cs],
                                     ti.d.n0 + ch * geo.c_cols, row0 + w * rows_w, c_policy);
+#else
+              ptx::tma_load_2d(cbuf + (size_t)cs * kCSlotBytes + w * rows_w * geo.c_swz, mapC, &sh->cfull[cs],
+                               ti.d.n0 + ch * geo.c_cols, row0 + w * rows_w);
+#endif
           } else {
             ptx::mbar_arrive(&sh->cfull[cs]);
           }
@@ -570,6 +594,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     const int half = (warp - 8) >> 2;
     const bool storer = half == 0;
     const uint64_t c_policy = ptx::policy_evict_first();
+    (void)c_policy;
     int re = 0, cs = 0, pending = -1;
     uint32_t rph = 0, cph = 0, t = 0;
     AccRing acc_ring;
@@ -672,7 +697,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 #else
           if (live && col0 < n8) {
 #endif
+#if VB_CSTORE_HINT
             ptx::tma_store_2d_hint(mapC, cb + r0 * geo.c_swz, col0, row0 + r0, c_policy);
+#else
+            ptx::tma_store_2d(mapC, cb + r0 * geo.c_swz, col0, row0 + r0);
+#endif
           }
           ptx::bulk_commit();
           if (pending >= 0) {
