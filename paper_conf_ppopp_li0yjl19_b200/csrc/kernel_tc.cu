@@ -64,6 +64,10 @@ constexpr int kPageBytes = 8192;
 #ifndef VB_AB_HINT
 #define VB_AB_HINT 0      // experiment: A/B loads marked L2 evict-last
 #endif
+#ifndef VB_NGRAN
+#define VB_NGRAN 16
+#endif
+constexpr int kNGran = VB_NGRAN;          // MMA N granularity per CTA for edge tiles (power of 2)
 constexpr int kPages = VB_PAGES;           // 144 KB of A/B staging (default)
 constexpr int kSlots = 16;                 // k-blocks in flight (bounded by pages anyway)
 constexpr int kCSlots = VB_CSLOTS;
@@ -125,6 +129,20 @@ enum TraceSlot {
 
 __device__ __forceinline__ int geo_BY(uint16_t g) { return (g & 0xFF) * 16; }
 __device__ __forceinline__ int geo_BX(uint16_t g) { return (g >> 8) * 16; }
+
+// MMA width of a tile: a tile at the right edge of its GEMM computes only the columns up to N,
+// rounded up to kNGran per CTA (a pair tile splits them evenly: CTA r supplies B columns
+// n0 + r * n/2 ..).  The columns past it are never stored, so tensor time on them is waste.
+__device__ __forceinline__ int mma_cols(int BX, int N, int n0, bool pair) {
+  const int g = pair ? 2 * kNGran : kNGran;
+  const int cols = min(BX, N - n0);
+  return min(BX, (cols + g - 1) & ~(g - 1));
+}
+// C chunks of a tile that hold any column < N (the epilogue and C producer skip the rest)
+__device__ __forceinline__ int live_chunks(const TcGeom &geo, int N, int n0) {
+  const int cols = min(geo.BX, N - n0);
+  return min(geo.c_chunks, (cols + geo.c_cols - 1) >> (__ffs(geo.c_cols) - 1));
+}
 
 // TMEM accumulator ring: tile t takes BX/32 contiguous 32-column units starting at `head`
 // (never wrapping); the MMA warp and the epilogue run this same function over the same tile
@@ -385,6 +403,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
         const int BXc = PAIR ? BX / 2 : BX;
         const TcGeom geo = tc_geom(BY, BXc);
+        const int Nh = mma_cols(BX, ti.d.N, ti.d.n0, PAIR) / (PAIR ? 2 : 1);   // B columns per CTA
         const uint8_t *maps = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128);
         // out-of-bounds box rows cost L2 bandwidth even though TMA zero-fills them: the last
         // row-tile uses the row-tail map, the last k-block the K-tail map, and B boxes that lie
@@ -395,18 +414,18 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           return rows <= 0 ? 0 : (rows < BY ? (rows + 7) / 8 * 8 : BY);
         };
         auto b_boxes_of = [&](int r) {
-          const int cols = ti.d.N - (ti.d.n0 + r * BXc);
+          const int cols = min(Nh, ti.d.N - (ti.d.n0 + r * Nh));
           const int bw = geo.b_swz / 2;                  // a power of two: shift, not divide
           return cols <= 0 ? 0 : min(geo.b_boxes, (cols + bw - 1) >> (__ffs(bw) - 1));
         };
-        const int row0 = ti.d.m0 + (int)rank * BY, col0 = ti.d.n0 + (int)rank * BXc;
+        const int row0 = ti.d.m0 + (int)rank * BY, col0 = ti.d.n0 + (int)rank * Nh;
         const int a_box_rows = a_box_rows_of((int)rank);
         const bool a_tail = a_box_rows != BY;
         const uint8_t *mapA = maps + (a_tail ? MAP_A_TAIL : MAP_A) * 128;
         const int b_boxes = b_boxes_of((int)rank);
         const int ksteps_last = (ti.d.flags >> 8) & 7;
         const int a_pages = BY * kBK * 2 / kPageBytes;
-        const int need = a_pages + (BXc * kBK * 2 + kPageBytes - 1) / kPageBytes;
+        const int need = a_pages + (Nh * kBK * 2 + kPageBytes - 1) / kPageBytes;
         for (int kb = 0; kb < ti.d.kblocks; ++kb, ++kbg) {
           int start = head, take = need;
           if (start + need > kPages) {          // never wrap a k-block around the ring end
@@ -502,7 +521,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         ++inflight;
         ptx::tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(start * kAccUnit);
-        const uint32_t idesc = ptx::idesc_f16((uint32_t)AB_FMT, BY, BX);
+        const uint32_t idesc = ptx::idesc_f16((uint32_t)AB_FMT, BY, mma_cols(BX, ti.d.N, ti.d.n0, PAIR));
         const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
         const uint32_t a_bytes = (uint32_t)(PAIR ? BY / 2 : BY) * kBK * 2;
         for (int kb = 0; kb < ti.d.kblocks; ++kb) {
@@ -562,7 +581,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const int row0 = ti.d.m0 + (int)rank * BY;
         const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C * 128;
         const bool load = ti.beta != 0.f;
-        for (int ch = 0; ch < geo.c_chunks; ++ch) {
+        const int nch = live_chunks(geo, ti.d.N, ti.d.n0);
+        for (int ch = 0; ch < nch; ++ch) {
           VB_TWAIT(T_CPROD_CEMPTY, ptx::mbar_wait(&sh->cempty[cs], cph ^ 1u));
           if (load) {
             // the C map's box is one epilogue quarter's sub-box (BY/4 rows); skip rows >= M
@@ -715,7 +735,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       };
 
       uint32_t a0[32];
-      const int nch = geo.c_chunks;
+      const int nch = live_chunks(geo, ti.d.N, ti.d.n0);
       if (!has_acc) {
 #pragma unroll
         for (int i = 0; i < 32; ++i) a0[i] = 0u;   // K == 0: C = beta * C
