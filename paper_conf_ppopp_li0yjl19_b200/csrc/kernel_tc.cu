@@ -463,6 +463,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             }
           }
           // box 0 = A, boxes 1..b_boxes = B; box i goes to producer (i + kbg) % kProducers
+          if (ptx::elect_lane0())
           for (int i = (int)((pid - kbg) % kProducers + kProducers) % kProducers; i <= b_boxes; i += kProducers) {
             if (i == 0 && a_box_rows == 0) continue;
             uint8_t *dst = i == 0 ? sa : sb + (i - 1) * kBK * geo.b_swz;
@@ -524,6 +525,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const uint32_t idesc = ptx::idesc_f16((uint32_t)AB_FMT, BY, mma_cols(BX, ti.d.N, ti.d.n0, PAIR));
         const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
         const uint32_t a_bytes = (uint32_t)(PAIR ? BY / 2 : BY) * kBK * 2;
+        // descriptors of K step 0; step kk adds 32 B (A) / 16 rows * b_swz (B) to the start
+        // address field (bits 0-13, address >> 4)
+        const uint64_t adesc0 = ptx::smem_desc(0, 16, 1024, 2);
+        const uint64_t bdesc0 = ptx::smem_desc(0, kBK * geo.b_swz, 8 * geo.b_swz, blayout);
+        const uint32_t b_step = (uint32_t)geo.b_swz;    // (16 * b_swz) >> 4
         for (int kb = 0; kb < ti.d.kblocks; ++kb) {
           VB_TWAIT(T_MMA_FULL, ptx::mbar_wait(&sh->full[slot], sph));
           ptx::tc_fence_after();
@@ -531,34 +537,35 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           const uint32_t sa = ptx::smem_u32(pages + (size_t)sh->slot_page[slot] * kPageBytes);
           const uint32_t sb = sa + a_bytes;
           const int ksteps = (kb == ti.d.kblocks - 1 && ((ti.d.flags >> 8) & 7)) ? ((ti.d.flags >> 8) & 7) : kBK / 16;
+          const uint64_t adesc = adesc0 | (uint64_t)(sa >> 4);
+          const uint64_t bdesc = bdesc0 | (uint64_t)(sb >> 4);
+          if (ptx::elect_lane0()) {
 #pragma unroll
-          for (int kk = 0; kk < kBK / 16; ++kk) {
-            if (kk >= ksteps) break;          // K tail: the B rows past the last step are not loaded
-            // A: K-major, 128-B swizzle, 8-row atoms 1024 B apart; K step of 16 = +32 B.
-            const uint64_t adesc = ptx::smem_desc(sa + kk * 32, 16, 1024, 2);
-            // B: MN-major, b_swz swizzle; 8-row (K) atoms 8*b_swz apart (SBO), MN blocks of
-            // b_swz/2 elements 64*b_swz apart (LBO); K step of 16 rows = +16*b_swz bytes.
-            const uint64_t bdesc = ptx::smem_desc(sb + kk * 16 * geo.b_swz, kBK * geo.b_swz, 8 * geo.b_swz, blayout);
+            for (int kk = 0; kk < kBK / 16; ++kk) {
+              if (kk >= ksteps) break;          // K tail: the B rows past the last step are not loaded
 #ifndef VB_EXP_NOMMA
-            if (PAIR)
-              ptx::mma_f16_ss_pair(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
-            else
-              ptx::mma_f16_ss(d_tmem, adesc, bdesc, idesc, (kb | kk) != 0 ? 1u : 0u);
+              if (PAIR)
+                ptx::mma_f16_ss_pair(d_tmem, adesc + 2u * kk, bdesc + b_step * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
+              else
+                ptx::mma_f16_ss(d_tmem, adesc + 2u * kk, bdesc + b_step * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
 #else
-            (void)adesc; (void)bdesc; (void)idesc; (void)d_tmem;
+              (void)adesc; (void)bdesc; (void)idesc; (void)d_tmem;
 #endif
+            }
+            if (PAIR)
+              ptx::mma_commit_pair(&sh->empty[slot]);   // frees the k-block's pages in both CTAs
+            else
+              ptx::mma_commit(&sh->empty[slot]);      // frees the k-block's pages when the MMAs retire
           }
-          if (PAIR)
-            ptx::mma_commit_pair(&sh->empty[slot]);   // frees the k-block's pages in both CTAs
-          else
-            ptx::mma_commit(&sh->empty[slot]);      // frees the k-block's pages when the MMAs retire
           VB_TADD(T_MMA_ISSUE);
           advance(slot, sph, kSlots);
         }
-        if (PAIR)
-          ptx::mma_commit_pair(&sh->tfull[e]);
-        else
-          ptx::mma_commit(&sh->tfull[e]);           // accumulator ready for the epilogue
+        if (ptx::elect_lane0()) {
+          if (PAIR)
+            ptx::mma_commit_pair(&sh->tfull[e]);
+          else
+            ptx::mma_commit(&sh->tfull[e]);         // accumulator ready for the epilogue
+        }
       }
     }
   } else if (warp == 2 || warp == 3) {
@@ -584,7 +591,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const int nch = live_chunks(geo, ti.d.N, ti.d.n0);
         for (int ch = 0; ch < nch; ++ch) {
           VB_TWAIT(T_CPROD_CEMPTY, ptx::mbar_wait(&sh->cempty[cs], cph ^ 1u));
-          if (load) {
+          if (load && ptx::elect_lane0()) {
             // the C map's box is one epilogue quarter's sub-box (BY/4 rows); skip rows >= M
             const int rows_w = BY / 4;
             int nsub = 0;
@@ -711,7 +718,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         // group have read their smem" always covers the previous chunk's slot.
         VB_TWAIT(T_EPI_FENCEBAR, ptx::fence_proxy_async_smem(); ptx::named_bar_sync(1 + q, 64));
         VB_T0();
-        if (storer && lane == 0) {
+        if (storer && lane == 0 && ptx::elect_lane0()) {
 #ifdef VB_EXP_NOSTORE
           if (false) {
 #else

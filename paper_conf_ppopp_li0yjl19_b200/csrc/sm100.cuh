@@ -267,5 +267,17 @@ __device__ __forceinline__ uint32_t swz(uint32_t off, int swz_bytes) {
   return off ^ (((off >> 7) & (uint32_t)(swz_bytes / 16 - 1)) << 4);
 }
 
+// elect.sync over lane 0 alone: for code that only lane 0 runs.  Inside the elected region the
+// compiler knows a single thread is active, so values feeding tcgen05 / TMA instructions go to
+// uniform registers directly instead of through an ELECT / R2UR.BROADCAST / BRA.U.ANY loop
+// per instruction.
+__device__ __forceinline__ bool elect_lane0() {
+  uint32_t p;
+  asm volatile(
+      "{\n.reg .pred P;\nelect.sync _|P, 1;\nselp.u32 %0, 1, 0, P;\n}\n"
+      : "=r"(p));
+  return p != 0;
+}
+
 }  // namespace ptx
 }  // namespace vb
