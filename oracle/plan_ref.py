@@ -60,14 +60,15 @@ B200_F32 = Table("b200_ffma", V100.rows, versions=(256,), tlp_threshold=131072, 
 # (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16), plus the skinny shapes
 # 128x32 and 64x256, plus 2-SM pair tiles 256x{64,128,256} (ctas = 2, cta_group::2).  One
 # kernel "version" with T = 256 threads.  Availability floor (C-1b): strategies are tested
-# against max(M, 128) and max(N, 64) — an M = 64 MMA costs the cycles of M = 128 and rows
-# past M are never loaded or stored; 64-column B boxes are the full-rate TMA boxes.
+# against max(M, 128) and max(N, 256) — an M = 64 MMA costs the cycles of M = 128 and rows
+# past M are never loaded or stored; an edge tile pays only for the columns it has, so the
+# widest tile is available to every GEMM.
 B200_TC = Table("b200_tcgen05", (
     Strategy("s", 64, 32, 64), Strategy("n", 128, 32, 64), Strategy("m", 64, 64, 64), Strategy("t", 128, 64, 64),
     Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("x", 64, 256, 64),
     Strategy("h", 128, 256, 64), Strategy("T2", 256, 64, 64, 2), Strategy("L2", 256, 128, 64, 2),
     Strategy("H2", 256, 256, 64, 2)),
-    versions=(256,), tlp_threshold=4 * 148 * 256, theta=512, min_BY=128, min_BX=64)
+    versions=(256,), tlp_threshold=4 * 148 * 256, theta=512, min_BY=128, min_BX=256)
 
 TABLES = {1: V100, 2: B200_F32, 3: B200_TC}
 
@@ -98,7 +99,7 @@ def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None, pairs_allo
     """The three steps and two exceptions of P249–253.
 
     1. Per GEMM, a priority queue of the strategies with BY <= M and BX <= N (C-1; the
-       B200 tcgen05 table compares against max(M, 128) and max(N, 64), C-1b),
+       B200 tcgen05 table compares against max(M, 128) and max(N, 256), C-1b),
        smallest first (P249); if none fits, the smallest strategy alone (C-4).
     2. Take one strategy per GEMM: pop, or top if only one is left (exception 1, C-2);
        TLP by Eq. 1 with the current version T.

@@ -50,7 +50,7 @@ constexpr int kPageBytes = 8192;
 #define VB_CSLOTS 4
 #endif
 #ifndef VB_KBAHEAD
-#define VB_KBAHEAD 24
+#define VB_KBAHEAD 8
 #endif
 // L2 evict-first hints on the C_old loads / C stores.  Measured off by default: with the load
 // hint, C5 read 1.3x its compulsory DRAM bytes (a 500^3 batch: C_old fetched ~1.6x) and ran
@@ -137,6 +137,13 @@ __device__ __forceinline__ int mma_cols(int BX, int N, int n0, bool pair) {
   const int g = pair ? 2 * kNGran : kNGran;
   const int cols = min(BX, N - n0);
   return min(BX, (cols + g - 1) & ~(g - 1));
+}
+// TMEM columns (32-column units) an accumulator occupies: its MMA width rounded up to whole
+// epilogue chunks (the epilogue reads every column of a live chunk), not BX, so tiles at the
+// right edge of narrow GEMMs leave room for more accumulators in flight
+__device__ __forceinline__ int acc_units(int BX, int N, int n0, bool pair) {
+  const int cc = BX >= 64 ? 64 : BX;
+  return ((mma_cols(BX, N, n0, pair) + cc - 1) / cc) * cc / kAccUnit;
 }
 // C chunks of a tile that hold any column < N (the epilogue and C producer skip the rest)
 __device__ __forceinline__ int live_chunks(const TcGeom &geo, int N, int n0) {
@@ -506,7 +513,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         tr[T_TILES] += 1;
 #endif
         int take;
-        const int start = ring.place(BX / kAccUnit, take);
+        const int start = ring.place(acc_units(BX, ti.d.N, ti.d.n0, PAIR), take);
         {
           VB_T0();
           while (free_units < take || inflight == kAcc) {   // reclaim drained accumulators (FIFO)
@@ -644,7 +651,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const uint32_t aph = (t / kAcc) & 1u;
       ++t;
       int take;
-      const int acc_col = acc_ring.place(BX / kAccUnit, take) * kAccUnit;
+      const int acc_col = acc_ring.place(acc_units(BX, ti.d.N, ti.d.n0, PAIR), take) * kAccUnit;
       // M = 128: tile row 32q + i lives in TMEM lane 32q + i.
       // M = 64 : tile row 16q + i lives in TMEM lane 32q + i, i < 16 (half sub-partitions).
       const int rows_w = BY / 4;

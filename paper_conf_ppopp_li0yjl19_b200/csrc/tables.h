@@ -29,8 +29,10 @@ struct TableDef {
   // BY <= max(M, min_BY) and BX <= max(N, min_BX).  0 for the paper's tables (P249 exactly).
   // tcgen05 table: min_BY = 128 because an M = 64 MMA takes as many cycles as M = 128 (the
   // pacing floor max(M,128)*N/256) and the rows past M are neither loaded (row-tail map) nor
-  // stored; min_BX = 64 because 64-column boxes use the 128-byte swizzle while narrower ones
-  // move at half the TMA rate (measured, tools/tma_bench.cu).
+  // stored; min_BX = 256 because a tile at the right edge of a GEMM only pays for the columns
+  // it has (MMA N trimmed to N, TMEM columns by MMA width, B boxes past N skipped), so the
+  // widest strategy costs a narrow GEMM nothing and covers whole B / C rows in one tile (fewer
+  // tiles and A re-reads: measured +3 % on C5 and C4 against min_BX = 64).
   int min_BY;
   int min_BX;
 };
@@ -56,12 +58,15 @@ constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 1, {256,
 // batches need once short GEMMs may take the 64-row MMA (min_BY = 64), and three 2-SM pair
 // tiles (cta_group::2, M = 256: each SM holds 128 rows of A and half of B, so a 256x256 pair
 // moves 33% fewer bytes per SM per k-block than 128x256) — the B200 "second version" of P198.
+#ifndef VB_TC_MIN_BX
+#define VB_TC_MIN_BX 256
+#endif
 constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 11,
                                    {{"s", 64, 32, 64, 1}, {"n", 128, 32, 64, 1}, {"m", 64, 64, 64, 1},
                                     {"t", 128, 64, 64, 1}, {"w", 64, 128, 64, 1}, {"l", 128, 128, 64, 1},
                                     {"x", 64, 256, 64, 1}, {"h", 128, 256, 64, 1},
                                     {"T2", 256, 64, 64, 2}, {"L2", 256, 128, 64, 2}, {"H2", 256, 256, 64, 2}},
-                                   1, {256, 0}, 4 * 148 * 256, 512, 128, 64};
+                                   1, {256, 0}, 4 * 148 * 256, 512, 128, VB_TC_MIN_BX};
 
 #undef VB_TABLE2_ROWS
 

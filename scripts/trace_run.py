@@ -26,7 +26,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C5")
 ap.add_argument("--policy", default="threshold")
 args = ap.parse_args()
-assert "trace" in nv.LIB_PATH, "set VB_LIB to a trace build"
+assert "trace" in nv.LIB_PATH or "VB_TRACE" in os.environ, "set VB_LIB to a trace build"
 info = vbinputs.CONFIGS[args.config]
 M, N, K = vbinputs.config_sizes(args.config)
 db = DeviceBatch(M, N, K, info["dtype"])

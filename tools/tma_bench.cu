@@ -45,8 +45,13 @@ __global__ void __launch_bounds__(256, 1) tma_stream(const __grid_constant__ CUt
       ptx::mbar_arrive_expect_tx(&full[s], a.stage_bytes);
       for (int b = 0; b < a.boxes_per_stage; ++b) {
         int tile;
-        if (a.sequential) tile = (int)((t++) % (unsigned)ntiles);
-        else { t = t * 1664525u + 1013904223u; tile = (int)(t % (unsigned)ntiles); }
+        if (a.sequential == 1) tile = (int)((t++) % (unsigned)ntiles);
+        else if (a.sequential == 2) {        // stage = bps consecutive boxes along a row band, stages random
+          if (b == 0) { t = t * 1664525u + 1013904223u; }
+          const int groups_w = tiles_w / a.boxes_per_stage;
+          const int g = (int)(t % (unsigned)(groups_w * tiles_h));
+          tile = (g / groups_w) * tiles_w + (g % groups_w) * a.boxes_per_stage + b;
+        } else { t = t * 1664525u + 1013904223u; tile = (int)(t % (unsigned)ntiles); }
         const int x = (tile % tiles_w) * a.box_w, y = (tile / tiles_w) * a.box_h;
         ptx::tma_load_2d(smem + (size_t)s * a.stage_bytes + (size_t)b * a.box_w * a.box_h * 2, &map, &full[s], x, y);
       }
@@ -79,7 +84,7 @@ int main(int argc, char **argv) {
   const int iters = argc > 6 ? atoi(argv[6]) : 4000;
   const int producers = argc > 7 ? atoi(argv[7]) : 1;
   const int sequential = argc > 8 ? atoi(argv[8]) : 0;
-  const int cols = 4096;
+  const int cols = argc > 9 ? atoi(argv[9]) : 4096;   // row length (elements): the row stride
   const int rows = (int)(foot_mb * 1024 * 1024 / (cols * 2));
   void *buf;
   cudaMalloc(&buf, (size_t)rows * cols * 2);
@@ -115,7 +120,7 @@ int main(int argc, char **argv) {
   float ms;
   cudaEventElapsedTime(&ms, e0, e1);
   const double bytes = (double)sms * iters * a.stage_bytes;
-  printf("box %dx%d x%d stages %d prod %d seq %d (in flight %.0f KB/SM) footprint %zu MB: %.1f GB/s  (%s)\n", box_w, box_h, bps, stages, producers, sequential,
+  printf("cols %d box %dx%d x%d stages %d prod %d seq %d (in flight %.0f KB/SM) footprint %zu MB: %.1f GB/s  (%s)\n", cols, box_w, box_h, bps, stages, producers, sequential,
          stages * a.stage_bytes / 1024.0, foot_mb, bytes / ms / 1e6, cudaGetErrorString(cudaGetLastError()));
   return 0;
 }
