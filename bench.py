@@ -309,7 +309,7 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
         "value": flops_all / (step_ms_max * 1e-3) / 1e12,
         "kernel_tflops": flops_all / (kern_ms_max * 1e-3) / 1e12,
         "roofline": roofline_for(dtype, flops, nbytes, kern_ms * 1e-3, peaks),
-        "plan": pinfo, "l2": "flushed (512 MB write) between steps" if small else
+        "plan": pinfo, "policy_chosen": {0: "threshold", 1: "binary", 2: "none"}.get(plan.policy(), "?"), "l2": "flushed (512 MB write) between steps" if small else
         f"inputs ({db.arena_bytes() / 1e9:.1f} GB per rank) >> L2 (126 MB); no flush",
         "launches": pinfo["launches_per_exec"] * steps, "clocks": clk, "batch_rank": int(db.batch),
     }
@@ -388,7 +388,8 @@ def main_ours(args):
             aux[cfg] = {"workload": workload_desc(cfg, args), "dtype": r["dtype"], "value": round(r["value"], 3),
                         "kernel_tflops": round(r["kernel_tflops"], 3), "ms_per_step": round(r["step_ms"], 4),
                         "plan_ms": round(r["plan_ms"], 2), "roofline": _round(r["roofline"]),
-                        "n_tiles": r["plan"]["n_tiles"], "n_blocks": r["plan"]["n_blocks"], "l2": r["l2"]}
+                        "n_tiles": r["plan"]["n_tiles"], "n_blocks": r["plan"]["n_blocks"], "l2": r["l2"],
+                        "policy": r["policy_chosen"]}
             del d2, p2
             torch.cuda.empty_cache()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -411,7 +412,8 @@ def main_ours(args):
         "config": {"workload": f"{args.config}: {workload_desc(args.config, args)}", "batch": int(
             len(vbinputs.config_sizes(args.config, nb=args.nb if args.config == 'C3' else 1)[0])),
             "parallelism": f"gemm-sharded x{world} (LPT on 2MNK, no data-path collective)" if world > 1 else
-            "single GPU", "policy": args.policy, "table": "b200_tcgen05" if res["dtype"] != "f32" else "b200_ffma",
+            "single GPU", "policy": args.policy if args.policy != "auto" else
+            f"auto (random forest, P272-274) -> {res['policy_chosen']}", "table": "b200_tcgen05" if res["dtype"] != "f32" else "b200_ffma",
             "l2": res["l2"], "plan_ms": round(res["plan_ms"], 2), "n_tiles_rank0": res["plan"]["n_tiles"],
             "n_blocks_rank0": res["plan"]["n_blocks"], "kernel_ms": round(res["kernel_ms"], 4),
             "kernel_tflops": round(res["kernel_tflops"], 3)},
@@ -468,7 +470,7 @@ def main(argv=None):
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", default="C5", choices=["C1", "C2", "C3", "C4", "C5"])
-    ap.add_argument("--policy", default="threshold", choices=["threshold", "binary", "none"])
+    ap.add_argument("--policy", default="auto", choices=["auto", "threshold", "binary", "none"])
     ap.add_argument("--nb", type=int, default=1, help="image batch for C3")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--e2e-steps", type=int, default=3)

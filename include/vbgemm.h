@@ -50,16 +50,21 @@ typedef enum { VB_F32 = 0, VB_BF16 = 1, VB_F16 = 2 } vb_dtype;   /* one dtype pe
 
 /* Batching policy (§5): THRESHOLD = TLP first (P261), BINARY = ILP first (P263-270),
  * NONE = one tile per block (the un-batched baseline, P259 "a thread block is
- * responsible for a single tile"). */
-typedef enum { VB_BATCH_THRESHOLD = 0, VB_BATCH_BINARY = 1, VB_BATCH_NONE = 2 } vb_policy;
+ * responsible for a single tile"), AUTO = on-line choice between THRESHOLD and BINARY by
+ * the random forest over (mean M, mean N, mean K, batch size) (P272-274), trained offline
+ * on B200 (reading C-25); vb_plan_policy reports the choice. */
+typedef enum {
+  VB_BATCH_THRESHOLD = 0, VB_BATCH_BINARY = 1, VB_BATCH_NONE = 2, VB_BATCH_AUTO = 3
+} vb_policy;
 
 /* Strategy tables.
  *  VB_TABLE_V100        PAPER.md Table 2 (P204-214) with the V100 constants (P290):
  *                       TLP threshold 65536, theta 256, versions T = 256 / 128.
  *  VB_TABLE_B200_FFMA   Table 2 shapes for the fp32 FFMA kernel, B200 constants.
  *  VB_TABLE_B200_TC     tcgen05 table (bf16/fp16): 64x32, 128x32, 64x64, 128x64, 64x128,
- *                       128x128, 64x256, 128x256 C tiles, BK = 64, T = 256; availability
- *                       tested against max(M, 64) x max(N, 32) (the 64-row MMA floor).
+ *                       128x128, 64x256, 128x256 C tiles and 2-SM pair tiles 256x{64,128,256},
+ *                       BK = 64, T = 256; availability tested against max(M, 128) x max(N, 256)
+ *                       (reading C-1b).
  *  VB_TABLE_DEFAULT     B200_FFMA for VB_F32, B200_TC for VB_BF16 / VB_F16. */
 typedef enum {
   VB_TABLE_DEFAULT = 0, VB_TABLE_V100 = 1, VB_TABLE_B200_FFMA = 2, VB_TABLE_B200_TC = 3
@@ -150,6 +155,29 @@ vb_status vb_exec_bound(vb_plan_t plan, const float *alpha, const float *beta, v
  * ------------------------------------------------------------------------------------ */
 vb_status vb_plan_info(vb_plan_t plan, int64_t *n_tiles, int64_t *n_blocks,
                        int64_t *workspace_bytes, int32_t *version_T, int32_t *launches_per_exec);
+
+/* vb_plan_policy — the batching policy the plan was built with (VB_BATCH_AUTO resolved to
+ * THRESHOLD or BINARY; -1 for a plan from vb_plan_from_schedule). */
+vb_status vb_plan_policy(vb_plan_t plan, int32_t *policy);
+
+/* ------------------------------------------------------------------------------------
+ * vb_plan_tune — "for the case where the batch size and the size of each matrix are fixed
+ * ... we can try both two batching heuristics and choose the better one" (P272).
+ * Plans the batch with THRESHOLD and with BINARY batching (same arguments as
+ * vb_plan_vbatched), runs each once to warm up and then `reps` times on `stream` with the
+ * caller's DEVICE buffers (as vb_exec_vbatched), times them with CUDA events, keeps the
+ * faster plan (ties keep THRESHOLD) and destroys the other.  *out is bound to A, B, C.
+ *  ms   nullable HOST float[2]: mean ms per run of THRESHOLD and BINARY.
+ * SYNCHRONISES `stream`.  C is used as scratch: it is overwritten (1 + reps) times per
+ * candidate and holds an unspecified value on return.  Errors as vb_plan_vbatched /
+ * vb_exec_vbatched; VB_ERR_UNSUPPORTED for device < 0.
+ * ------------------------------------------------------------------------------------ */
+vb_status vb_plan_tune(int device, vb_dtype dt, int32_t batch,
+                       const int32_t *M, const int32_t *N, const int32_t *K,
+                       const int32_t *lda, const int32_t *ldb, const int32_t *ldc,
+                       const vb_tuning *tuning, const void *const *A, const void *const *B,
+                       void *const *C, const float *alpha, const float *beta, int32_t reps,
+                       void *stream, vb_plan_t *out, float *ms);
 
 /* vb_plan_export — the five auxiliary arrays of §6 (HOST outputs, sized by vb_plan_info):
  *   block_ptr[n_blocks+1], tile_gemm/tile_y/tile_x[n_tiles], gemm_strategy[batch]

@@ -14,6 +14,8 @@ Contents
 * ``plan_ref``  — tiling engine (§4, P245–255, Eq. 1), tile enumeration (P133–135, P157),
                   threshold / binary batching (§5, P259–270, Eq. 5), five-array encoding
                   (§6, P282–284, Fig. 6/7) and the LPT GEMM->rank sharder (BASELINE.json).
+* ``forest_ref`` — the on-line batching-policy selector (random forest, §5, P272–274),
+                  evaluated on trees that are a B200 platform constant (reading C-25).
 * ``checks``    — normwise error, coverage map and plan invariants.
 
 Parity status: every function is pinned (see DESIGN.md §3 and tests/test_oracle_*.py) except

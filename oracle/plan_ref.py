@@ -54,7 +54,7 @@ V100 = Table("v100_table2", (
 # B200 FFMA (fp32) profile: the Table 2 shapes and sub-tiles are an FFMA design and are
 # kept; the platform constants are re-set for 148 SMs and only the 256-thread version is
 # offered (calibrated on B200, reading C-22).
-B200_F32 = Table("b200_ffma", V100.rows, versions=(256,), tlp_threshold=131072, theta=256)
+B200_F32 = Table("b200_ffma", V100.rows, versions=(256,), tlp_threshold=4 * 148 * 256, theta=64)
 
 # B200 tcgen05 (bf16/fp16) profile: C-tile shapes sized for tcgen05.mma
 # (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16), plus the skinny shapes
@@ -68,7 +68,7 @@ B200_TC = Table("b200_tcgen05", (
     Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("x", 64, 256, 64),
     Strategy("h", 128, 256, 64), Strategy("T2", 256, 64, 64, 2), Strategy("L2", 256, 128, 64, 2),
     Strategy("H2", 256, 256, 64, 2)),
-    versions=(256,), tlp_threshold=4 * 148 * 256, theta=512, min_BY=128, min_BX=256)
+    versions=(256,), tlp_threshold=148 * 256, theta=64, min_BY=128, min_BX=256)
 
 TABLES = {1: V100, 2: B200_F32, 3: B200_TC}
 

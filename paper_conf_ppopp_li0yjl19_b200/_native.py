@@ -18,7 +18,7 @@ HEADER = os.path.join(os.path.dirname(HERE), "include", "vbgemm.h")
 
 VB_OK, VB_ERR_INVALID_ARG, VB_ERR_ALIGNMENT, VB_ERR_UNSUPPORTED, VB_ERR_OOM, VB_ERR_CUDA, VB_ERR_INTERNAL = range(7)
 VB_F32, VB_BF16, VB_F16 = 0, 1, 2
-VB_BATCH_THRESHOLD, VB_BATCH_BINARY, VB_BATCH_NONE = 0, 1, 2
+VB_BATCH_THRESHOLD, VB_BATCH_BINARY, VB_BATCH_NONE, VB_BATCH_AUTO = 0, 1, 2, 3
 VB_TABLE_DEFAULT, VB_TABLE_V100, VB_TABLE_B200_FFMA, VB_TABLE_B200_TC = 0, 1, 2, 3
 DTYPE_CODE = {"f32": VB_F32, "bf16": VB_BF16, "f16": VB_F16}
 
@@ -58,13 +58,16 @@ lib.vb_plan_info.argtypes = [_vp, _i64p, _i64p, _i64p, _i32p, _i32p]
 lib.vb_plan_export.argtypes = [_vp, _i32p, _i32p, _i32p, _i32p, _i32p]
 lib.vb_plan_tiler_trace.argtypes = [_vp, ctypes.c_int32, _i64p, _i32p, _i32p]
 lib.vb_plan_destroy.argtypes = [_vp]
+lib.vb_plan_policy.argtypes = [_vp, _i32p]
+lib.vb_plan_tune.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int32] + [_i32p] * 6 + \
+    [_P(vb_tuning), _vp, _vp, _vp, _vp, _vp, ctypes.c_int32, _vp, _P(_vp), _P(ctypes.c_float)]
 lib.vb_shard_lpt.argtypes = [ctypes.c_int32, _i32p, _i32p, _i32p, ctypes.c_int32, _i32p]
 lib.vb_fill_uniform_batch.argtypes = [ctypes.c_int, ctypes.c_int32, _vp, _vp, _vp, _vp, _vp, ctypes.c_uint64,
                                       ctypes.c_int32, ctypes.c_int64, _vp]
 lib.vb_fill_alpha_beta.argtypes = [ctypes.c_int32, _vp, ctypes.c_uint64, _vp, _vp, _vp]
 lib.vb_device_info.argtypes = [ctypes.c_int, _i32p, _i32p, _i32p]
 for _f in ("vb_plan_vbatched", "vb_plan_from_schedule", "vb_exec_vbatched", "vb_plan_bind", "vb_exec_bound", "vb_plan_info", "vb_plan_export",
-           "vb_plan_tiler_trace", "vb_plan_destroy", "vb_shard_lpt", "vb_fill_uniform_batch", "vb_fill_alpha_beta",
+           "vb_plan_tiler_trace", "vb_plan_destroy", "vb_plan_policy", "vb_plan_tune", "vb_shard_lpt", "vb_fill_uniform_batch", "vb_fill_alpha_beta",
            "vb_device_info"):
     getattr(lib, _f).restype = ctypes.c_int
 
@@ -121,6 +124,12 @@ class Plan:
         return dict(n_tiles=nt.value, n_blocks=nb.value, workspace_bytes=ws.value, version_T=vt.value,
                     launches_per_exec=nl.value)
 
+    def policy(self) -> int:
+        """The batching policy the plan was built with (AUTO resolved; -1 for a user schedule)."""
+        v = ctypes.c_int32()
+        check(lib.vb_plan_policy(self.handle, ctypes.byref(v)))
+        return v.value
+
     def export(self) -> dict:
         inf = self.info()
         bp = np.zeros(inf["n_blocks"] + 1, np.int32)
@@ -162,6 +171,22 @@ def plan_vbatched(M, N, K, lda, ldb, ldc, dtype: str = "bf16", policy: int = VB_
     check(lib.vb_plan_vbatched(int(device), DTYPE_CODE[dtype], batch, *[_ptr(a, _i32p) for a in arrs], int(policy),
                                ctypes.byref(tun), ctypes.byref(h)))
     return Plan(h.value, batch, dtype)
+
+
+def plan_tune(M, N, K, lda, ldb, ldc, A_ptrs: int, B_ptrs: int, C_ptrs: int, alpha: int, beta: int,
+              dtype: str = "bf16", device: int = 0, reps: int = 3, stream: int = 0, table_id: int = 0,
+              tlp_threshold: int = 0, theta: int = 0):
+    """vb_plan_tune: time THRESHOLD and BINARY on the given DEVICE buffers and keep the faster
+    (P272).  Synchronises the stream; C is overwritten.  Returns (plan, [ms_threshold, ms_binary])."""
+    arrs = [_i32(a) for a in (M, N, K, lda, ldb, ldc)]
+    batch = len(arrs[0])
+    tun = vb_tuning(table_id, tlp_threshold, theta)
+    h = ctypes.c_void_p()
+    ms = (ctypes.c_float * 2)()
+    check(lib.vb_plan_tune(int(device), DTYPE_CODE[dtype], batch, *[_ptr(a, _i32p) for a in arrs], ctypes.byref(tun),
+                           _vp(A_ptrs), _vp(B_ptrs), _vp(C_ptrs), _vp(alpha), _vp(beta), int(reps), _vp(stream),
+                           ctypes.byref(h), ms))
+    return Plan(h.value, batch, dtype), [ms[0], ms[1]]
 
 
 def plan_from_schedule(M, N, K, lda, ldb, ldc, gemm_row, version_T, block_ptr, tile_gemm, tile_y, tile_x,

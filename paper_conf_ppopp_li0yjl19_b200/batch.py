@@ -122,6 +122,13 @@ class DeviceBatch:
                                 device=self.device.index or 0, table_id=table_id, tlp_threshold=tlp_threshold,
                                 theta=theta)
 
+    def plan_tune(self, reps: int = 3, stream=None, **tuning):
+        """vb_plan_tune on this batch's buffers (C is overwritten): (plan, [ms_threshold, ms_binary])."""
+        s = torch.cuda.current_stream(self.device) if stream is None else stream
+        return nv.plan_tune(self.M, self.N, self.K, self.lda, self.ldb, self.ldc, self.pA.data_ptr(),
+                            self.pB.data_ptr(), self.pC.data_ptr(), self.alpha.data_ptr(), self.beta.data_ptr(),
+                            self.dtype, device=self.device.index or 0, reps=reps, stream=s.cuda_stream, **tuning)
+
     def run(self, plan: nv.Plan, stream=None) -> None:
         """vb_exec_vbatched: bind this batch's pointers and run (two launches on the tc path)."""
         s = torch.cuda.current_stream(self.device) if stream is None else stream

@@ -16,6 +16,8 @@
 
 #include "../../include/vbgemm.h"
 #include "plan_types.h"
+#include "forest.h"
+#include "forest_b200.h"
 #include "planner.h"
 #include "tables.h"
 
@@ -325,8 +327,14 @@ extern "C" vb_status vb_plan_vbatched(int device, vb_dtype dt, int32_t batch, co
     *out = nullptr;
     vb_status st = validate_shapes(dt, batch, M, N, K, lda, ldb, ldc);
     if (st != VB_OK) return st;
-    if (policy != VB_BATCH_THRESHOLD && policy != VB_BATCH_BINARY && policy != VB_BATCH_NONE)
+    if (policy != VB_BATCH_THRESHOLD && policy != VB_BATCH_BINARY && policy != VB_BATCH_NONE &&
+        policy != VB_BATCH_AUTO)
       return fail(VB_ERR_INVALID_ARG, "unknown policy %d", (int)policy);
+    if (policy == VB_BATCH_AUTO) {   // online selection by the B200 random forest (P272-274)
+      float x[4];
+      forest_features(M, N, K, batch, x);
+      policy = forest_select(dt == VB_F32 ? kForestF32 : kForestTc, x) ? VB_BATCH_BINARY : VB_BATCH_THRESHOLD;
+    }
     const TableDef *t = resolve_table(dt, tuning ? tuning->table_id : 0);
     if (!t) return fail(VB_ERR_INVALID_ARG, "unknown table id %d", tuning ? tuning->table_id : -1);
     if (device >= 0 && !table_runs_on(t, dt))
@@ -543,6 +551,60 @@ extern "C" vb_status vb_exec_vbatched(vb_plan_t p, const void *const *A, const v
   vb_status st = vb_plan_bind(p, A, B, C, stream);
   if (st != VB_OK) return st;
   return vb_exec_bound(p, alpha, beta, stream);
+}
+
+extern "C" vb_status vb_plan_policy(vb_plan_t p, int32_t *policy) {
+  if (!p || !policy) return fail(VB_ERR_INVALID_ARG, "null argument");
+  *policy = p->policy;
+  return VB_OK;
+}
+
+extern "C" vb_status vb_plan_tune(int device, vb_dtype dt, int32_t batch, const int32_t *M, const int32_t *N,
+                                  const int32_t *K, const int32_t *lda, const int32_t *ldb, const int32_t *ldc,
+                                  const vb_tuning *tuning, const void *const *A, const void *const *B, void *const *C,
+                                  const float *alpha, const float *beta, int32_t reps, void *stream, vb_plan_t *out,
+                                  float *ms) {
+  if (!out) return fail(VB_ERR_INVALID_ARG, "out is null");
+  *out = nullptr;
+  if (device < 0) return fail(VB_ERR_UNSUPPORTED, "tuning needs a device");
+  if (reps < 1) reps = 1;
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess) return cuda_fail(g.err, "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const vb_policy cand[2] = {VB_BATCH_THRESHOLD, VB_BATCH_BINARY};
+  vb_plan_t plans[2] = {nullptr, nullptr};
+  float t[2] = {0.f, 0.f};
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  vb_status st = VB_OK;
+  cudaError_t ce = cudaEventCreate(&e0);
+  if (ce == cudaSuccess) ce = cudaEventCreate(&e1);
+  if (ce != cudaSuccess) st = cuda_fail(ce, "cudaEventCreate");
+  for (int c = 0; c < 2 && st == VB_OK; ++c) {
+    st = vb_plan_vbatched(device, dt, batch, M, N, K, lda, ldb, ldc, cand[c], tuning, &plans[c]);
+    if (st == VB_OK) st = vb_exec_vbatched(plans[c], A, B, C, alpha, beta, stream);   // warm-up, binds
+    if (st != VB_OK) break;
+    ce = cudaEventRecord(e0, s);
+    for (int r = 0; r < reps && st == VB_OK; ++r) st = vb_exec_bound(plans[c], alpha, beta, stream);
+    if (ce == cudaSuccess) ce = cudaEventRecord(e1, s);
+    if (ce == cudaSuccess) ce = cudaEventSynchronize(e1);
+    if (ce == cudaSuccess) ce = cudaEventElapsedTime(&t[c], e0, e1);
+    if (st == VB_OK && ce != cudaSuccess) st = cuda_fail(ce, "timing");
+  }
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  if (st != VB_OK) {
+    vb_plan_destroy(plans[0]);
+    vb_plan_destroy(plans[1]);
+    return st;
+  }
+  const int keep = t[1] < t[0] ? 1 : 0;    // ties keep threshold (TLP first)
+  vb_plan_destroy(plans[1 - keep]);   // each plan keeps its own maps, bound by its warm-up run
+  if (ms) {
+    ms[0] = t[0] / reps;
+    ms[1] = t[1] / reps;
+  }
+  *out = plans[keep];
+  return VB_OK;
 }
 
 extern "C" vb_status vb_plan_info(vb_plan_t p, int64_t *n_tiles, int64_t *n_blocks, int64_t *workspace_bytes,

@@ -50,7 +50,9 @@ constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 1
 // sm_100a), threshold re-set for 148 SMs (reading C-22).  Calibrated on B200: the 128-thread
 // version (16x8 sub-tiles, 255 registers, 8 warps per SM) is 13% slower than the 256-thread
 // version at two CTAs per SM on C2, so this profile offers the 256-thread version only.
-constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 1, {256, 0}, 131072, 256, 0, 0};
+// Constants calibrated on B200 over the Fig. 8/9 grid + C1/C2 (scripts/calibrate_grid.py,
+// profiles/calibration_grid_f32_r01.json): TLP threshold 4 * 148 * 256, theta 64.
+constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 1, {256, 0}, 4 * 148 * 256, 64, 0, 0};
 
 // B200 tcgen05 profile (bf16/fp16): C tiles for tcgen05.mma with M in {64,128}; BK = 64 =
 // one 128-byte swizzled row of bf16; 256 threads per tile in Eq. 1.  Besides the paper's
@@ -61,12 +63,15 @@ constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 1, {256,
 #ifndef VB_TC_MIN_BX
 #define VB_TC_MIN_BX 256
 #endif
+// Constants calibrated on B200 over the Fig. 8/9 grid + C3/C4/C5 (scripts/calibrate_grid.py,
+// profiles/calibration_grid_bf16_r01.json): TLP threshold 148 * 256 (one tile per SM: the
+// persistent kernel overlaps the tiles of an SM), theta 64 (one BK = 64 k-block).
 constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 11,
                                    {{"s", 64, 32, 64, 1}, {"n", 128, 32, 64, 1}, {"m", 64, 64, 64, 1},
                                     {"t", 128, 64, 64, 1}, {"w", 64, 128, 64, 1}, {"l", 128, 128, 64, 1},
                                     {"x", 64, 256, 64, 1}, {"h", 128, 256, 64, 1},
                                     {"T2", 256, 64, 64, 2}, {"L2", 256, 128, 64, 2}, {"H2", 256, 256, 64, 2}},
-                                   1, {256, 0}, 4 * 148 * 256, 512, 128, VB_TC_MIN_BX};
+                                   1, {256, 0}, 148 * 256, 64, 128, VB_TC_MIN_BX};
 
 #undef VB_TABLE2_ROWS
 

@@ -291,3 +291,31 @@ def test_memory_bound_batch_keeps_one_sm_tiles():
     assert not pr.pairs_allowed(M, N, K)
     M, N, K = vbinputs.config_sizes("C4")
     assert pr.pairs_allowed(M, N, K)
+
+
+# ------------------------------------------------------------------ policy selection (P272-274)
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_auto_policy_parity(dtype):
+    """VB_BATCH_AUTO (random-forest choice) runs the chosen heuristic and stays exact."""
+    rng = np.random.default_rng(3)
+    M, N, K = (rng.integers(1, 300, 40) for _ in range(3))
+    db, plan = _run(M, N, K, dtype, vb.VB_BATCH_AUTO)
+    assert plan.policy() in (vb.VB_BATCH_THRESHOLD, vb.VB_BATCH_BINARY)
+    check_batch(db, range(db.batch), SEED, "random")
+    _padding_untouched(db)
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_plan_tune_keeps_faster_and_is_exact(dtype):
+    """vb_plan_tune (P272: try both heuristics on a fixed batch, keep the better one)."""
+    rng = np.random.default_rng(4)
+    M, N, K = (rng.integers(16, 400, 64) for _ in range(3))
+    db = DeviceBatch(M, N, K, dtype)
+    db.fill(SEED, "random")
+    plan, ms = db.plan_tune(reps=3)
+    assert ms[0] > 0 and ms[1] > 0
+    assert plan.policy() == (vb.VB_BATCH_BINARY if ms[1] < ms[0] else vb.VB_BATCH_THRESHOLD)
+    db.fill(SEED, "random")          # tuning used C as scratch: restore C_old, then run the kept plan
+    db.run(plan)
+    torch.cuda.synchronize()
+    check_batch(db, range(db.batch), SEED, "random")
