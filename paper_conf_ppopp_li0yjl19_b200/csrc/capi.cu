@@ -77,6 +77,7 @@ struct vb_plan {
   TileDesc *d_tiles = nullptr;      // tensor-core path: one record per slot
   std::vector<TileDesc> tiles;
   uint8_t *d_tmaps = nullptr;
+  int32_t *d_order = nullptr;       // FFMA path: launch order of the blocks, heaviest first
   int32_t *d_counter = nullptr;     // pair kernel [0] work-list, [1] finished CTAs; 1-SM kernel [2], [3]
   int n_pair_blocks = 0;            // blocks [0, n_pair_blocks) hold 2-SM pair tiles
   int sm_count = 0;
@@ -189,6 +190,8 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   off = align_up(off + std::max<size_t>(p->gemms.size(), 1) * sizeof(GemmParam), 256);
   const size_t o_td = off;
   if (tc) off = align_up(off + std::max<size_t>(p->tiles.size(), 1) * sizeof(TileDesc), 256);
+  const size_t o_or = off;
+  if (!tc) off = align_up(off + std::max<size_t>(p->block_ptr.size(), 1) * sizeof(int32_t), 256);
   const size_t o_ct = off;
   off = align_up(off + 256, 256);
   const size_t o_tm = off;
@@ -205,6 +208,7 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   p->d_gemms = reinterpret_cast<GemmParam *>(base + o_gp);
   p->d_counter = reinterpret_cast<int32_t *>(base + o_ct);
   p->d_tiles = tc ? reinterpret_cast<TileDesc *>(base + o_td) : nullptr;
+  p->d_order = tc ? nullptr : reinterpret_cast<int32_t *>(base + o_or);
   p->d_tmaps = tc ? base + o_tm : nullptr;
 
   if (!tc) {
@@ -212,6 +216,25 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(f32 kernel smem)");
   }
   std::vector<uint8_t> host(p->ws_bytes, 0);
+  if (!tc && p->block_ptr.size() > 1) {
+    // The FFMA kernel is launched with grid = Block_NUM (Fig. 7); the hardware hands out CTAs in
+    // index order, so CTA j runs block order[j], blocks sorted by estimated FMA work (tile area x
+    // K rounded to the kernel's 32-wide k-slice, plus a per-tile constant), heaviest first: the
+    // longest blocks start in the first wave instead of forming the tail (LPT).  The plan itself
+    // (block_ptr, slots) is unchanged.
+    const int nb = (int)p->block_ptr.size() - 1;
+    std::vector<int64_t> work((size_t)nb, 0);
+    for (int b = 0; b < nb; ++b)
+      for (int32_t s = p->block_ptr[b]; s < p->block_ptr[b + 1]; ++s) {
+        const GemmParam &g = p->gemms[p->slots[(size_t)s].gemm];
+        const StrategyRow &r = p->table->rows[g.row & 0xFF];
+        work[(size_t)b] += (int64_t)r.BY * r.BX * (cdiv64(g.K, 32) * 32 + 64);
+      }
+    std::vector<int32_t> order((size_t)nb);
+    for (int b = 0; b < nb; ++b) order[(size_t)b] = b;
+    std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return work[(size_t)a] > work[(size_t)b]; });
+    memcpy(host.data() + o_or, order.data(), order.size() * sizeof(int32_t));
+  }
   memcpy(host.data() + o_bp, p->block_ptr.data(), p->block_ptr.size() * sizeof(int32_t));
   if (!p->slots.empty()) memcpy(host.data() + o_sl, p->slots.data(), p->slots.size() * sizeof(TileSlot));
   if (!p->gemms.empty()) memcpy(host.data() + o_gp, p->gemms.data(), p->gemms.size() * sizeof(GemmParam));
@@ -524,7 +547,7 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
   if (p->dt == VB_F32) {
     F32Args a{p->d_block_ptr, p->d_slots, p->d_gemms, reinterpret_cast<const float *const *>(p->bound_A),
               reinterpret_cast<const float *const *>(p->bound_B), reinterpret_cast<float *const *>(p->bound_C),
-              alpha, beta};
+              alpha, beta, p->d_order};
     e = launch_f32(a, n_blocks, p->tiling.version_T, s);
   } else {
     // 2-SM pair tiles first (clusters of 2 over blocks [0, n_pair)), then the 1-SM tiles

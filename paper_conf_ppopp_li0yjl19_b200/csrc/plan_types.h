@@ -34,6 +34,7 @@ struct F32Args {
   float *const *C;
   const float *alpha;
   const float *beta;
+  const int32_t *order;   // launch order: CTA j runs block order[j] (heaviest first; not part of the plan)
 };
 
 // Per tile slot, precomputed by the planner for the tensor-core kernel: the five arrays of
