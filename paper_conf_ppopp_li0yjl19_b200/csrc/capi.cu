@@ -9,6 +9,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <queue>
 #include <mutex>
 #include <new>
 #include <string>
@@ -23,6 +24,8 @@
 
 namespace vb {
 cudaError_t launch_f32(const F32Args &args, int n_blocks, int version_T, cudaStream_t stream);
+cudaError_t launch_f32_prep(uint8_t *tmaps, const void *const *A, const void *const *B, const GemmParam *gemms,
+                            int batch, cudaStream_t stream);
 cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
                            const GemmParam *gemms, int batch, int32_t *counter, cudaStream_t stream);
 cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, cudaStream_t stream);
@@ -77,7 +80,8 @@ struct vb_plan {
   TileDesc *d_tiles = nullptr;      // tensor-core path: one record per slot
   std::vector<TileDesc> tiles;
   uint8_t *d_tmaps = nullptr;
-  int32_t *d_order = nullptr;       // FFMA path: launch order of the blocks, heaviest first
+  int32_t *d_order = nullptr;       // FFMA path: claim order of the blocks, heaviest first
+  int f32_grid = 0;
   int32_t *d_counter = nullptr;     // pair kernel [0] work-list, [1] finished CTAs; 1-SM kernel [2], [3]
   int n_pair_blocks = 0;            // blocks [0, n_pair_blocks) hold 2-SM pair tiles
   int sm_count = 0;
@@ -121,12 +125,15 @@ static vb_status encode_2d(CUtensorMap *m, vb_dtype dt, void *addr, uint64_t inn
                            uint32_t box_inner, uint32_t box_outer, int swz_bytes) {
   auto enc = get_encode();
   if (!enc) return fail(VB_ERR_CUDA, "cuTensorMapEncodeTiled entry point unavailable");
-  const CUtensorMapDataType t = dt == VB_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  const CUtensorMapDataType t = dt == VB_BF16   ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                : dt == VB_F16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                                               : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
   cuuint64_t dims[2] = {inner, outer};
-  cuuint64_t strides[1] = {ld_elems * 2};
+  cuuint64_t strides[1] = {ld_elems * (dt == VB_F32 ? 4 : 2)};
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t estr[2] = {1, 1};
-  CUresult r = enc(m, t, 2, addr, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_of(swz_bytes),
+  CUresult r = enc(m, t, 2, addr, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   swz_bytes ? swizzle_of(swz_bytes) : CU_TENSOR_MAP_SWIZZLE_NONE,
 #ifndef VB_L2PROMO
 #define VB_L2PROMO CU_TENSOR_MAP_L2_PROMOTION_L2_256B
 #endif
@@ -190,12 +197,17 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   off = align_up(off + std::max<size_t>(p->gemms.size(), 1) * sizeof(GemmParam), 256);
   const size_t o_td = off;
   if (tc) off = align_up(off + std::max<size_t>(p->tiles.size(), 1) * sizeof(TileDesc), 256);
+#ifndef VB_F32_CTAS_PER_SM
+#define VB_F32_CTAS_PER_SM 2
+#endif
+  const int n_blocks = (int)p->block_ptr.size() - 1;
+  p->f32_grid = tc ? 0 : std::min(n_blocks, VB_F32_CTAS_PER_SM * p->sm_count);
   const size_t o_or = off;
-  if (!tc) off = align_up(off + std::max<size_t>(p->block_ptr.size(), 1) * sizeof(int32_t), 256);
+  if (!tc) off = align_up(off + (size_t)std::max(n_blocks, 1) * sizeof(int32_t), 256);
   const size_t o_ct = off;
   off = align_up(off + 256, 256);
   const size_t o_tm = off;
-  if (tc) off = align_up(off + (size_t)p->batch * kMapsPerGemm * 128, 256);
+  off = align_up(off + (size_t)p->batch * (tc ? kMapsPerGemm : kF32MapsPerGemm) * 128, 256);
   p->ws_bytes = off;
   e = cudaMalloc(&p->d_ws, p->ws_bytes);
   if (e != cudaSuccess) {
@@ -209,29 +221,28 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   p->d_counter = reinterpret_cast<int32_t *>(base + o_ct);
   p->d_tiles = tc ? reinterpret_cast<TileDesc *>(base + o_td) : nullptr;
   p->d_order = tc ? nullptr : reinterpret_cast<int32_t *>(base + o_or);
-  p->d_tmaps = tc ? base + o_tm : nullptr;
+  p->d_tmaps = base + o_tm;
 
   if (!tc) {
     e = f32_configure();
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(f32 kernel smem)");
   }
   std::vector<uint8_t> host(p->ws_bytes, 0);
-  if (!tc && p->block_ptr.size() > 1) {
-    // The FFMA kernel is launched with grid = Block_NUM (Fig. 7); the hardware hands out CTAs in
-    // index order, so CTA j runs block order[j], blocks sorted by estimated FMA work (tile area x
-    // K rounded to the kernel's 32-wide k-slice, plus a per-tile constant), heaviest first: the
-    // longest blocks start in the first wave instead of forming the tail (LPT).  The plan itself
-    // (block_ptr, slots) is unchanged.
-    const int nb = (int)p->block_ptr.size() - 1;
-    std::vector<int64_t> work((size_t)nb, 0);
-    for (int b = 0; b < nb; ++b)
+  if (!tc && n_blocks > 0) {
+    // Execution order of the FFMA kernel: its persistent CTAs claim blocks through an atomic
+    // counter in the order order[0], order[1], ...: blocks sorted by estimated FMA work (tile
+    // area x K rounded to the kernel's 32-wide k-slice, plus a per-tile constant), heaviest
+    // first, so the longest blocks start first instead of forming the tail (LPT).  The plan
+    // itself (block_ptr, slots: the batching engine's output) is unchanged.
+    std::vector<int64_t> work((size_t)n_blocks, 0);
+    for (int b = 0; b < n_blocks; ++b)
       for (int32_t s = p->block_ptr[b]; s < p->block_ptr[b + 1]; ++s) {
         const GemmParam &g = p->gemms[p->slots[(size_t)s].gemm];
         const StrategyRow &r = p->table->rows[g.row & 0xFF];
         work[(size_t)b] += (int64_t)r.BY * r.BX * (cdiv64(g.K, 32) * 32 + 64);
       }
-    std::vector<int32_t> order((size_t)nb);
-    for (int b = 0; b < nb; ++b) order[(size_t)b] = b;
+    std::vector<int32_t> order((size_t)n_blocks);
+    for (int b = 0; b < n_blocks; ++b) order[(size_t)b] = b;
     std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return work[(size_t)a] > work[(size_t)b]; });
     memcpy(host.data() + o_or, order.data(), order.size() * sizeof(int32_t));
   }
@@ -282,6 +293,23 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
                        (uint32_t)g.c_cols, (uint32_t)(BYc / 4), g.c_swz);
         if (st != VB_OK) return st;
       }
+    }
+  }
+  if (!tc) {
+    // fp32 maps: A box = 32 floats (one 128-byte swizzled row) x BY rows; B box
+    // = min(BX, 32) floats x 32 rows, unswizzled.  Encoded with a placeholder address; bind
+    // patches the address.
+    CUtensorMap *maps = reinterpret_cast<CUtensorMap *>(host.data() + o_tm);
+    for (int i = 0; i < p->batch; ++i) {
+      if (M[i] == 0 || N[i] == 0 || K[i] == 0) continue;
+      const StrategyRow &s = p->table->rows[p->tiling.row[i]];
+      CUtensorMap *m = &maps[(size_t)kF32MapsPerGemm * i];
+      vb_status st = encode_2d(&m[0], p->dt, p->d_ws, (uint64_t)K[i], (uint64_t)M[i], (uint64_t)lda[i], 32,
+                               (uint32_t)s.BY, 128);
+      if (st != VB_OK) return st;
+      const uint32_t bw = (uint32_t)std::min(s.BX, 32);
+      st = encode_2d(&m[1], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)K[i], (uint64_t)ldb[i], bw, 32, 0);
+      if (st != VB_OK) return st;
     }
   }
   e = cudaMemcpy(p->d_ws, host.data(), p->ws_bytes, cudaMemcpyHostToDevice);
@@ -525,9 +553,13 @@ extern "C" vb_status vb_plan_bind(vb_plan_t p, const void *const *A, const void 
   p->bound_A = A;
   p->bound_B = B;
   p->bound_C = C;
-  if (p->batch == 0 || p->dt == VB_F32) return VB_OK;
+  if (p->batch == 0) return VB_OK;
   DeviceGuard g(p->device);
   if (g.err != cudaSuccess) return cuda_fail(g.err, "cudaSetDevice");
+  if (p->dt == VB_F32) {
+    cudaError_t e = launch_f32_prep(p->d_tmaps, A, B, p->d_gemms, p->batch, static_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? VB_OK : cuda_fail(e, "prep kernel launch");
+  }
   cudaError_t e = launch_tc_prep(p->d_tmaps, A, B, C, p->d_gemms, p->batch, p->d_counter,
                                  static_cast<cudaStream_t>(stream));
   return e == cudaSuccess ? VB_OK : cuda_fail(e, "prep kernel launch");
@@ -547,8 +579,8 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
   if (p->dt == VB_F32) {
     F32Args a{p->d_block_ptr, p->d_slots, p->d_gemms, reinterpret_cast<const float *const *>(p->bound_A),
               reinterpret_cast<const float *const *>(p->bound_B), reinterpret_cast<float *const *>(p->bound_C),
-              alpha, beta, p->d_order};
-    e = launch_f32(a, n_blocks, p->tiling.version_T, s);
+              alpha, beta, p->d_order, p->d_tmaps, p->d_counter, n_blocks};
+    e = launch_f32(a, p->f32_grid, p->tiling.version_T, s);
   } else {
     // 2-SM pair tiles first (clusters of 2 over blocks [0, n_pair)), then the 1-SM tiles
     const int n_pair = p->n_pair_blocks, n_single = n_blocks - n_pair;

@@ -34,8 +34,13 @@ struct F32Args {
   float *const *C;
   const float *alpha;
   const float *beta;
-  const int32_t *order;   // launch order: CTA j runs block order[j] (heaviest first; not part of the plan)
+  const int32_t *order;   // claim order of the blocks, heaviest first (execution detail, not part of the plan)
+  const void *tmaps;      // CUtensorMap[batch][kF32MapsPerGemm] (A, B), 128-byte aligned
+  int32_t *counter;       // [0] work-list counter, [1] finished CTAs (reset by the last CTA)
+  int32_t n_blocks;
 };
+// fp32 tensor maps per GEMM: A (box 32 x BY, 128-byte swizzle) and B (box min(BX,32) x 32).
+constexpr int kF32MapsPerGemm = 2;
 
 // Per tile slot, precomputed by the planner for the tensor-core kernel: the five arrays of
 // Fig. 6 joined with the per-GEMM sizes, so the kernel reads one 32-byte record per tile.

@@ -247,7 +247,7 @@ def test_bind_then_exec_bound_repeatedly(dtype):
         db.plan().exec_bound(db.alpha.data_ptr(), db.beta.data_ptr(), 0)   # never bound
 
 
-@pytest.mark.parametrize("dtype", ["bf16", "f16"])
+@pytest.mark.parametrize("dtype", ["bf16", "f16", "f32"])
 def test_rebind_alternating_buffers_never_uses_stale_descriptors(dtype):
     # one plan, two batches with identical shapes in different arenas; re-bind back and forth
     # (tensor maps are patched in place by the prep kernel) and check every result
