@@ -244,13 +244,22 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
     import paper_conf_ppopp_li0yjl19_b200 as vb
     from paper_conf_ppopp_li0yjl19_b200.batch import DeviceBatch
 
-    info = vbinputs.CONFIGS[cfg]
-    dtype, ab = info["dtype"], info["ab"]
-    nb = args.nb if cfg == "C3" else 1
-    M, N, K = vbinputs.config_sizes(cfg, nb=nb)
-    idx = shard_indices(M, N, K, world, rank, vb.shard_lpt)
     dev = torch.device("cuda", local)
-    db = DeviceBatch(M[idx], N[idx], K[idx], dtype, device=dev, gemm_ids=idx)
+    if cfg == "C3i":   # the C3 convolutions as implicit GEMMs (vb_plan_conv, NEXT-3)
+        from paper_conf_ppopp_li0yjl19_b200.batch import ConvBatch
+        dtype, ab = "bf16", "conv"
+        convs = vbinputs.googlenet_convs(nb=args.nb)
+        idx = np.asarray(shard_indices(np.array([1] * len(convs)), np.array([1] * len(convs)),
+                                       np.array([1] * len(convs)), world, rank, vb.shard_lpt)) if world > 1 else \
+            np.arange(len(convs))
+        db = ConvBatch([convs[i] for i in idx], dtype, device=dev, gemm_ids=idx)
+    else:
+        info = vbinputs.CONFIGS[cfg]
+        dtype, ab = info["dtype"], info["ab"]
+        nb = args.nb if cfg == "C3" else 1
+        M, N, K = vbinputs.config_sizes(cfg, nb=nb)
+        idx = shard_indices(M, N, K, world, rank, vb.shard_lpt)
+        db = DeviceBatch(M[idx], N[idx], K[idx], dtype, device=dev, gemm_ids=idx)
     db.fill(args.seed, ab)
     torch.cuda.synchronize(dev)
     t0 = time.perf_counter()
@@ -363,6 +372,9 @@ def run_e2e(db, plan, args, world, dist_device, flops_all, stream, dev):
 
 
 def workload_desc(cfg, args):
+    if cfg == "C3i":
+        return (f"the 54 GoogleNet inception branch convolutions as batched implicit GEMMs (TMA im2col, "
+                f"NHWC x HWIO, bf16, nb={args.nb}); algorithmic bytes = input + weights + output")
     d = vbinputs.CONFIGS[cfg]["desc"]
     return d + (f" (nb={args.nb})" if cfg == "C3" else "")
 
@@ -383,7 +395,7 @@ def main_ours(args):
     if world == 1 and not args.no_aux:
         del db, plan
         torch.cuda.empty_cache()
-        for cfg in [c for c in ("C2", "C3", "C4") if c != args.config]:
+        for cfg in [c for c in ("C2", "C3", "C3i", "C4") if c != args.config]:
             r, d2, p2 = run_config(cfg, args, world, rank, local, peaks, dist_device, headline=False)
             aux[cfg] = {"workload": workload_desc(cfg, args), "dtype": r["dtype"], "value": round(r["value"], 3),
                         "kernel_tflops": round(r["kernel_tflops"], 3), "ms_per_step": round(r["step_ms"], 4),

@@ -118,6 +118,42 @@ vb_status vb_plan_from_schedule(int device, vb_dtype dt, int32_t batch,
                                 const int32_t *tile_x, vb_plan_t *out);
 
 /* ------------------------------------------------------------------------------------
+ * vb_plan_conv — a batch of 2-D convolutions run as batched IMPLICIT GEMMs (SURVEY.md §8(f)
+ * NEXT-3): "GEMM is the core of convolution ... the im2col approach transforms the
+ * convolution into a GEMM" with M = #filters, N = H*W*images, K = Cin*kh*kw (PAPER.md P45,
+ * P338-352).  Here the im2col matrix is never materialised: the kernel's A-operand producer
+ * loads it tile by tile with TMA im2col-mode copies straight from the NHWC input, so each
+ * convolution reads its input, weights and output once.  Orientation (transposed against
+ * P45 so that the output is NHWC): the GEMM is
+ *     Y[p][co] = alpha * sum_{kh,kw,ci} X[n][h+kh-pad][w+kw-pad][ci] * Wt[kh][kw][ci][co]
+ *                + beta * Y[p][co]
+ * with p = (n*Hout + h)*Wout + w the output pixel (GEMM row, M = nb*Hout*Wout), co the output
+ * channel (GEMM column, N = Cout) and K = KH*KW*Cin ordered (kh, kw, ci); X outside the
+ * image reads as 0.  Hout = H + 2*pad - KH + 1, Wout = W + 2*pad - KW + 1 (stride 1,
+ * dilation 1; "same" convolution for pad = (KH-1)/2).
+ *  dt       VB_BF16 or VB_F16 (tensor-core path; fp32 accumulation).
+ *  desc     HOST vb_conv_desc[batch].  Layouts, all row-major, element strides:
+ *           X  (exec's A[i]): NHWC, nb x H x W x Cin, dense (pixel stride Cin).
+ *           Wt (exec's B[i]): HWIO, the (KH*KW*Cin) x Cout GEMM B matrix, row stride ldb.
+ *           Y  (exec's C[i]): NHWC output, (nb*Hout*Wout) x Cout, row stride ldc -- an
+ *              inception module's branches write into one concatenated tensor by passing
+ *              its channel offset in the pointer and the total channel count as ldc.
+ *  Constraints (else VB_ERR_INVALID_ARG / VB_ERR_ALIGNMENT): sizes >= 1, KH == KW <= 8,
+ *           0 <= pad < KH, Hout, Wout >= 1, Cin % 8 == 0, ldb >= Cout, ldc >= Cout,
+ *           ldb % 8 == 0, ldc % 8 == 0 (16-byte rows), nb*H*W*Cin < 2^31.
+ * The tiling and batching engines run on (M, N, K) exactly as vb_plan_vbatched (1-SM
+ * strategies only); execution is vb_exec_vbatched / vb_plan_bind + vb_exec_bound with the
+ * pointer arrays above.  Ownership and errors as vb_plan_vbatched.
+ * ------------------------------------------------------------------------------------ */
+typedef struct {
+  int32_t nb, H, W, Cin, Cout, KH, KW, pad;
+  int32_t ldb, ldc;
+} vb_conv_desc;
+
+vb_status vb_plan_conv(int device, vb_dtype dt, int32_t batch, const vb_conv_desc *desc,
+                       vb_policy policy, const vb_tuning *tuning, vb_plan_t *out);
+
+/* ------------------------------------------------------------------------------------
  * vb_exec_vbatched — enqueue the batched GEMM on `stream`.
  *  A, B     DEVICE arrays [batch] of DEVICE pointers to the matrices (16-byte aligned).
  *  C        DEVICE array  [batch] of DEVICE pointers (16-byte aligned), read+written.

@@ -16,6 +16,8 @@ Contents
                   (§6, P282–284, Fig. 6/7) and the LPT GEMM->rank sharder (BASELINE.json).
 * ``forest_ref`` — the on-line batching-policy selector (random forest, §5, P272–274),
                   evaluated on trees that are a B200 platform constant (reading C-25).
+* ``conv_ref``  — stride-1 zero-padded 2-D convolution in fp64 (NHWC x HWIO), the definition
+                  behind the implicit-GEMM convolution path (NEXT-3, P45, P338–352).
 * ``checks``    — normwise error, coverage map and plan invariants.
 
 Parity status: every function is pinned (see DESIGN.md §3 and tests/test_oracle_*.py) except

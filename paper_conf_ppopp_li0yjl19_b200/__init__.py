@@ -12,7 +12,7 @@ The compute path is libvbgemm.so only; importing without it raises ImportError.
 """
 from ._native import (  # noqa: F401
     Plan, VbError, check, device_info, fill_alpha_beta, fill_uniform_batch, header_symbols, lib, plan_from_schedule,
-    plan_tune, plan_vbatched, shard_lpt, version,
+    plan_conv, plan_tune, plan_vbatched, shard_lpt, version,
     VB_BATCH_AUTO, VB_BATCH_BINARY, VB_BATCH_NONE, VB_BATCH_THRESHOLD,
     VB_TABLE_B200_FFMA, VB_TABLE_B200_TC, VB_TABLE_DEFAULT, VB_TABLE_V100,
     VB_OK, VB_ERR_ALIGNMENT, VB_ERR_CUDA, VB_ERR_INTERNAL, VB_ERR_INVALID_ARG, VB_ERR_OOM, VB_ERR_UNSUPPORTED,

@@ -33,6 +33,10 @@ class vb_tuning(ctypes.Structure):
     _fields_ = [("table_id", ctypes.c_int32), ("tlp_threshold", ctypes.c_int64), ("theta", ctypes.c_int32)]
 
 
+class vb_conv_desc(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in ("nb", "H", "W", "Cin", "Cout", "KH", "KW", "pad", "ldb", "ldc")]
+
+
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: run `python paper_conf_ppopp_li0yjl19_b200/build.py` "
                       "(or __graft_entry__.build()) first; there is no fallback path")
@@ -51,6 +55,8 @@ lib.vb_plan_vbatched.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int32] + [
     [ctypes.c_int, _P(vb_tuning), _P(_vp)]
 lib.vb_plan_from_schedule.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int32] + [_i32p] * 6 + \
     [ctypes.c_int32, _i32p, ctypes.c_int32, ctypes.c_int32, _i32p, _i32p, _i32p, _i32p, _P(_vp)]
+lib.vb_plan_conv.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int32, _P(vb_conv_desc), ctypes.c_int,
+                             _P(vb_tuning), _P(_vp)]
 lib.vb_exec_vbatched.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp]
 lib.vb_plan_bind.argtypes = [_vp, _vp, _vp, _vp, _vp]
 lib.vb_exec_bound.argtypes = [_vp, _vp, _vp, _vp]
@@ -171,6 +177,20 @@ def plan_vbatched(M, N, K, lda, ldb, ldc, dtype: str = "bf16", policy: int = VB_
     check(lib.vb_plan_vbatched(int(device), DTYPE_CODE[dtype], batch, *[_ptr(a, _i32p) for a in arrs], int(policy),
                                ctypes.byref(tun), ctypes.byref(h)))
     return Plan(h.value, batch, dtype)
+
+
+def plan_conv(convs, dtype: str = "bf16", policy: int = VB_BATCH_THRESHOLD, device: int = 0, table_id: int = 0,
+              tlp_threshold: int = 0, theta: int = 0) -> Plan:
+    """vb_plan_conv: convs = sequence of dicts with keys nb, H, W, Cin, Cout, KH, KW, pad, ldb, ldc."""
+    arr = (vb_conv_desc * max(len(convs), 1))()
+    for i, c in enumerate(convs):
+        for k, _ in vb_conv_desc._fields_:
+            setattr(arr[i], k, int(c[k]))
+    tun = vb_tuning(table_id, tlp_threshold, theta)
+    h = ctypes.c_void_p()
+    check(lib.vb_plan_conv(int(device), DTYPE_CODE[dtype], len(convs), arr, int(policy), ctypes.byref(tun),
+                           ctypes.byref(h)))
+    return Plan(h.value, len(convs), dtype)
 
 
 def plan_tune(M, N, K, lda, ldb, ldc, A_ptrs: int, B_ptrs: int, C_ptrs: int, alpha: int, beta: int,

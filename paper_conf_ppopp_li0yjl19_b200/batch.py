@@ -142,3 +142,72 @@ class DeviceBatch:
     def run_bound(self, plan: nv.Plan, stream=None) -> None:
         s = torch.cuda.current_stream(self.device) if stream is None else stream
         plan.exec_bound(self.alpha.data_ptr(), self.beta.data_ptr(), s.cuda_stream)
+
+
+class ConvBatch(DeviceBatch):
+    """A batch of convolutions for vb_plan_conv (implicit GEMM, NEXT-3): per convolution an
+    NHWC input X (the exec call's A), HWIO weights (B, (KH*KW*Cin) x Cout, row stride ldb) and an
+    NHWC output (C, (nb*Hout*Wout) x Cout, row stride ldc).  Inputs are drawn by the same device
+    generator as GEMM batches: X is operand A with logical shape (nb*H*W) x Cin, the weights are
+    operand B with shape K x Cout, the output operand C."""
+
+    def __init__(self, convs, dtype: str = "bf16", device="cuda:0", gemm_ids=None):
+        self.convs = [dict(c) for c in convs]
+        for c in self.convs:
+            c["Hout"] = c["H"] + 2 * c["pad"] - c["KH"] + 1
+            c["Wout"] = c["W"] + 2 * c["pad"] - c["KW"] + 1
+        cv = self.convs
+        self.M = np.array([c["nb"] * c["Hout"] * c["Wout"] for c in cv], np.int64)
+        self.N = np.array([c["Cout"] for c in cv], np.int64)
+        self.K = np.array([c["KH"] * c["KW"] * c["Cin"] for c in cv], np.int64)
+        self.P = np.array([c["nb"] * c["H"] * c["W"] for c in cv], np.int64)     # input pixels
+        self.Cin = np.array([c["Cin"] for c in cv], np.int64)
+        self.batch = len(cv)
+        self.dtype = dtype
+        self.es = vbinputs.elem_size(dtype)
+        self.device = torch.device(device)
+        self.gemm_ids = np.arange(self.batch, dtype=np.int64) if gemm_ids is None else np.asarray(gemm_ids, np.int64)
+        self.lda = self.Cin.copy()                       # dense NHWC: pixel stride = Cin
+        self.ldb = vbinputs.padded_ld(self.N, dtype)
+        self.ldc = vbinputs.padded_ld(self.N, dtype)
+        for c, b, l in zip(cv, self.ldb, self.ldc):
+            c["ldb"], c["ldc"] = int(b), int(l)
+        td = TORCH_DTYPE[dtype]
+        self.offA, nA = _layout(self.P, self.Cin, self.lda, self.es)
+        self.offB, nB = _layout(self.K, self.N, self.ldb, self.es)
+        self.offC, nC = _layout(self.M, self.N, self.ldc, self.es)
+        self.A = torch.empty(nA, dtype=td, device=self.device)
+        self.B = torch.empty(nB, dtype=td, device=self.device)
+        self.C = torch.empty(nC, dtype=td, device=self.device)
+        es = self.es
+
+        def ptrs(arena, offs):
+            return torch.from_numpy(arena.data_ptr() + offs * es).to(self.device)
+
+        self.pA, self.pB, self.pC = ptrs(self.A, self.offA), ptrs(self.B, self.offB), ptrs(self.C, self.offC)
+        self.alpha = torch.ones(max(self.batch, 1), dtype=torch.float32, device=self.device)
+        self.beta = torch.zeros(max(self.batch, 1), dtype=torch.float32, device=self.device)
+        self.d_gemm_ids = torch.from_numpy(self.gemm_ids).to(self.device)
+        self._dims = {}
+
+    def algorithmic_bytes(self, beta_nonzero=True) -> int:
+        """Compulsory bytes of the convolutions: input + weights + output (+ old output if beta != 0);
+        the im2col matrix is never materialised."""
+        bn = np.ones(self.batch, bool) if beta_nonzero is True else np.asarray(beta_nonzero, bool)
+        mn = self.M * self.N
+        return int((self.es * (self.P * self.Cin + self.K * self.N) + self.es * mn * (1 + bn)).sum())
+
+    def _dim_arrays(self, which):
+        if which not in self._dims:
+            rows, cols, ld = {"A": (self.P, self.Cin, self.lda), "B": (self.K, self.N, self.ldb),
+                              "C": (self.M, self.N, self.ldc)}[which]
+            t = lambda a: torch.from_numpy(np.ascontiguousarray(a, np.int32)).to(self.device)  # noqa: E731
+            self._dims[which] = (t(rows), t(cols), t(ld), int((rows * cols).sum()))
+        return self._dims[which]
+
+    def a(self, g):
+        return self._view(self.A, self.offA[g], self.P[g], self.Cin[g], self.lda[g])
+
+    def plan(self, policy=nv.VB_BATCH_THRESHOLD, table_id=0, tlp_threshold=0, theta=0) -> nv.Plan:
+        return nv.plan_conv(self.convs, self.dtype, policy, device=self.device.index or 0, table_id=table_id,
+                            tlp_threshold=tlp_threshold, theta=theta)

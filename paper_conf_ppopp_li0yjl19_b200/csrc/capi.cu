@@ -82,6 +82,9 @@ struct vb_plan {
   uint8_t *d_tmaps = nullptr;
   int32_t *d_order = nullptr;       // FFMA path: claim order of the blocks, heaviest first
   int f32_grid = 0;
+  std::vector<ConvParam> conv;      // convolution plans (vb_plan_conv): one per GEMM, else empty
+  std::vector<vb_conv_desc> conv_desc;
+  ConvParam *d_conv = nullptr;
   int32_t *d_counter = nullptr;     // pair kernel [0] work-list, [1] finished CTAs; 1-SM kernel [2], [3]
   int n_pair_blocks = 0;            // blocks [0, n_pair_blocks) hold 2-SM pair tiles
   int sm_count = 0;
@@ -142,6 +145,34 @@ static vb_status encode_2d(CUtensorMap *m, vb_dtype dt, void *addr, uint64_t inn
     return fail(VB_ERR_INTERNAL, "cuTensorMapEncodeTiled failed (%d) dims %llu x %llu ld %llu box %u x %u", (int)r,
                 (unsigned long long)inner, (unsigned long long)outer, (unsigned long long)ld_elems, box_inner,
                 box_outer);
+  return VB_OK;
+}
+
+// im2col-mode map over an NHWC tensor (nb x H x W x Cin): boxes of `pixels` output pixels x 64
+// channels (128 bytes, 128-byte swizzle: the same smem layout as a tiled A box), traversal
+// bounding box of the window origins [-pad, W - 1 + pad - (KW - 1)] (same in H).
+static vb_status encode_im2col(CUtensorMap *m, vb_dtype dt, void *addr, const vb_conv_desc &c, uint32_t pixels) {
+  static PFN_cuTensorMapEncodeIm2col_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *q = nullptr;
+    cudaDriverEntryPointQueryResult r;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &q, cudaEnableDefault, &r) == cudaSuccess &&
+        r == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeIm2col_v12000>(q);
+  });
+  if (!fn) return fail(VB_ERR_CUDA, "cuTensorMapEncodeIm2col entry point unavailable");
+  const CUtensorMapDataType t = dt == VB_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  cuuint64_t dims[4] = {(cuuint64_t)c.Cin, (cuuint64_t)c.W, (cuuint64_t)c.H, (cuuint64_t)c.nb};
+  cuuint64_t strides[3] = {(cuuint64_t)c.Cin * 2, (cuuint64_t)c.W * c.Cin * 2, (cuuint64_t)c.H * c.W * c.Cin * 2};
+  int lower[2] = {-c.pad, -c.pad};
+  int upper[2] = {c.pad - (c.KW - 1), c.pad - (c.KH - 1)};
+  cuuint32_t estr[4] = {1, 1, 1, 1};
+  CUresult r = fn(m, t, 4, addr, dims, strides, lower, upper, 64, pixels, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  CU_TENSOR_MAP_SWIZZLE_128B, VB_L2PROMO, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS)
+    return fail(VB_ERR_INTERNAL, "cuTensorMapEncodeIm2col failed (%d) nb %d H %d W %d Cin %d k %d pad %d pixels %u",
+                (int)r, c.nb, c.H, c.W, c.Cin, c.KH, c.pad, pixels);
   return VB_OK;
 }
 
@@ -208,6 +239,8 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   off = align_up(off + 256, 256);
   const size_t o_tm = off;
   off = align_up(off + (size_t)p->batch * (tc ? kMapsPerGemm : kF32MapsPerGemm) * 128, 256);
+  const size_t o_cv = off;
+  if (!p->conv.empty()) off = align_up(off + p->conv.size() * sizeof(ConvParam), 256);
   p->ws_bytes = off;
   e = cudaMalloc(&p->d_ws, p->ws_bytes);
   if (e != cudaSuccess) {
@@ -222,6 +255,7 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   p->d_tiles = tc ? reinterpret_cast<TileDesc *>(base + o_td) : nullptr;
   p->d_order = tc ? nullptr : reinterpret_cast<int32_t *>(base + o_or);
   p->d_tmaps = base + o_tm;
+  p->d_conv = p->conv.empty() ? nullptr : reinterpret_cast<ConvParam *>(base + o_cv);
 
   if (!tc) {
     e = f32_configure();
@@ -250,6 +284,7 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   if (!p->slots.empty()) memcpy(host.data() + o_sl, p->slots.data(), p->slots.size() * sizeof(TileSlot));
   if (!p->gemms.empty()) memcpy(host.data() + o_gp, p->gemms.data(), p->gemms.size() * sizeof(GemmParam));
   if (tc && !p->tiles.empty()) memcpy(host.data() + o_td, p->tiles.data(), p->tiles.size() * sizeof(TileDesc));
+  if (!p->conv.empty()) memcpy(host.data() + o_cv, p->conv.data(), p->conv.size() * sizeof(ConvParam));
   if (tc) {
     e = tc_configure();
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(tc kernel smem)");
@@ -264,7 +299,18 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
       const TcGeom gb = tc_geom(BYc, s.BX / s.ctas);       // B boxes of this CTA's half
       CUtensorMap *m = &maps[(size_t)kMapsPerGemm * i];
       vb_status st;
-      if (K[i] > 0) {
+      if (!p->conv.empty()) {   // implicit GEMM: A = im2col(X) by TMA im2col copies, B = HWIO weights
+        const vb_conv_desc &c = p->conv_desc[(size_t)i];
+        st = encode_im2col(&m[MAP_A], p->dt, p->d_ws, c, (uint32_t)BYc);
+        if (st != VB_OK) return st;
+        if (M[i] % BYc) {
+          st = encode_im2col(&m[MAP_A_TAIL], p->dt, p->d_ws, c, (uint32_t)((M[i] % BYc + 7) / 8 * 8));
+          if (st != VB_OK) return st;
+        }
+        st = encode_2d(&m[MAP_B], p->dt, p->d_ws, (uint64_t)N[i], (uint64_t)K[i], (uint64_t)ldb[i],
+                       (uint32_t)(gb.b_swz / 2), 64, gb.b_swz);
+        if (st != VB_OK) return st;
+      } else if (K[i] > 0) {
         st = encode_2d(&m[MAP_A], p->dt, p->d_ws, (uint64_t)K[i], (uint64_t)M[i], (uint64_t)lda[i], 64,
                        (uint32_t)BYc, 128);
         if (st != VB_OK) return st;
@@ -362,11 +408,93 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
       // granule is stored directly
       const int last_chunk_end = d.n0 + s.BX;
       d.flags = (uint16_t)(((g.N & 7) != 0 && last_chunk_end > g.N && d.n0 < g.N) ? 1 : 0);
-      if (g.K % 64) d.flags |= (uint16_t)(((g.K % 64 + 15) / 16) << 8);   // MMA K-steps of the last k-block
+      if (!p->conv.empty()) {   // implicit GEMM: taps x channel blocks, every k-block full (zero-filled channels)
+        const ConvParam &c = p->conv[ts.gemm];
+        d.kblocks = g.K > 0 ? (g.K / c.Cin) * c.ncb : 0;
+        d.flags |= kFlagConv;
+      } else if (g.K % 64) {
+        d.flags |= (uint16_t)(((g.K % 64 + 15) / 16) << 8);   // MMA K-steps of the last k-block
+      }
       (void)geo;
     }
   }
   if (p->device >= 0) return upload(p, M, N, K, lda, ldb, ldc);
+  return VB_OK;
+}
+
+// Tiling engine + batching engine + descriptor upload for one batch (vb_plan_vbatched and
+// vb_plan_conv).  conv: nullptr, or the convolution of each GEMM (implicit GEMM; 1-SM only).
+static vb_status plan_impl(int device, vb_dtype dt, int32_t batch, const int32_t *M, const int32_t *N,
+                           const int32_t *K, const int32_t *lda, const int32_t *ldb, const int32_t *ldc,
+                           vb_policy policy, const vb_tuning *tuning, const vb_conv_desc *conv, vb_plan_t *out) {
+  if (policy != VB_BATCH_THRESHOLD && policy != VB_BATCH_BINARY && policy != VB_BATCH_NONE &&
+      policy != VB_BATCH_AUTO)
+    return fail(VB_ERR_INVALID_ARG, "unknown policy %d", (int)policy);
+  if (policy == VB_BATCH_AUTO) {   // online selection by the B200 random forest (P272-274)
+    float x[4];
+    forest_features(M, N, K, batch, x);
+    policy = forest_select(dt == VB_F32 ? kForestF32 : kForestTc, x) ? VB_BATCH_BINARY : VB_BATCH_THRESHOLD;
+  }
+  const TableDef *t = resolve_table(dt, tuning ? tuning->table_id : 0);
+  if (!t) return fail(VB_ERR_INVALID_ARG, "unknown table id %d", tuning ? tuning->table_id : -1);
+  if (device >= 0 && !table_runs_on(t, dt))
+    return fail(VB_ERR_UNSUPPORTED, "table %s has no kernel for this dtype", t->name);
+  const int64_t thr = (tuning && tuning->tlp_threshold > 0) ? tuning->tlp_threshold : t->tlp_threshold;
+  const int theta = (tuning && tuning->theta > 0) ? tuning->theta : t->theta;
+  vb_plan *p = new vb_plan();
+  p->device = device;
+  p->dt = dt;
+  p->batch = batch;
+  p->table = t;
+  p->policy = (int)policy;
+  if (conv) {
+    p->conv_desc.assign(conv, conv + batch);
+    p->conv.resize((size_t)batch);
+    for (int i = 0; i < batch; ++i) {
+      const vb_conv_desc &c = conv[i];
+      ConvParam &q = p->conv[(size_t)i];
+      q.Hout = c.H + 2 * c.pad - c.KH + 1;
+      q.Wout = c.W + 2 * c.pad - c.KW + 1;
+      q.Cin = c.Cin;
+      q.KW = c.KW;
+      q.pad = c.pad;
+      q.ncb = (c.Cin + 63) / 64;
+      q.pad_[0] = q.pad_[1] = 0;
+    }
+  }
+  p->tiling = tiling_engine(M, N, batch, *t, thr, !conv && pairs_allowed(M, N, K, batch, elem_bytes(dt)));
+  if (batch == 0) p->tiling.version_T = t->versions[0];
+  const std::vector<TileRec> all = enumerate_tiles(M, N, K, batch, p->tiling.row, *t);
+  if (all.size() > (size_t)INT32_MAX) {
+    delete p;
+    return fail(VB_ERR_INVALID_ARG, "more than 2^31 tiles");
+  }
+  // 2-SM pair tiles run in their own cluster kernel: batch them separately, pair blocks first.
+  std::vector<TileRec> tiles;
+  tiles.reserve(all.size());
+  for (const TileRec &r : all)
+    if (t->rows[p->tiling.row[r.gemm]].ctas == 2) tiles.push_back(r);
+  const size_t n_pair = tiles.size();
+  for (const TileRec &r : all)
+    if (t->rows[p->tiling.row[r.gemm]].ctas != 2) tiles.push_back(r);
+  Schedule sch;
+  sch.block_ptr.push_back(0);
+  for (int part = 0; part < 2; ++part) {
+    const std::vector<TileRec> sub(tiles.begin() + (part ? n_pair : 0), part ? tiles.end() : tiles.begin() + n_pair);
+    const Schedule sp = policy == VB_BATCH_THRESHOLD ? batch_threshold(sub, p->tiling.version_T, thr, theta)
+                        : policy == VB_BATCH_BINARY  ? batch_binary(sub, theta)
+                                                     : batch_none(sub);
+    const int32_t base = (int32_t)sch.slot_tile.size(), off = part ? (int32_t)n_pair : 0;
+    for (int32_t v : sp.slot_tile) sch.slot_tile.push_back(v + off);
+    for (size_t b = 1; b < sp.block_ptr.size(); ++b) sch.block_ptr.push_back(base + sp.block_ptr[b]);
+    if (part == 0) p->n_pair_blocks = (int)sch.block_ptr.size() - 1;
+  }
+  const vb_status st = finish_plan(p, M, N, K, lda, ldb, ldc, tiles, sch);
+  if (st != VB_OK) {
+    delete p;
+    return st;
+  }
+  *out = p;
   return VB_OK;
 }
 
@@ -378,60 +506,47 @@ extern "C" vb_status vb_plan_vbatched(int device, vb_dtype dt, int32_t batch, co
     *out = nullptr;
     vb_status st = validate_shapes(dt, batch, M, N, K, lda, ldb, ldc);
     if (st != VB_OK) return st;
-    if (policy != VB_BATCH_THRESHOLD && policy != VB_BATCH_BINARY && policy != VB_BATCH_NONE &&
-        policy != VB_BATCH_AUTO)
-      return fail(VB_ERR_INVALID_ARG, "unknown policy %d", (int)policy);
-    if (policy == VB_BATCH_AUTO) {   // online selection by the B200 random forest (P272-274)
-      float x[4];
-      forest_features(M, N, K, batch, x);
-      policy = forest_select(dt == VB_F32 ? kForestF32 : kForestTc, x) ? VB_BATCH_BINARY : VB_BATCH_THRESHOLD;
+    return plan_impl(device, dt, batch, M, N, K, lda, ldb, ldc, policy, tuning, nullptr, out);
+  } catch (const std::bad_alloc &) {
+    return fail(VB_ERR_OOM, "host allocation failed");
+  } catch (...) {
+    return fail(VB_ERR_INTERNAL, "unexpected exception");
+  }
+}
+
+extern "C" vb_status vb_plan_conv(int device, vb_dtype dt, int32_t batch, const vb_conv_desc *desc, vb_policy policy,
+                                  const vb_tuning *tuning, vb_plan_t *out) {
+  try {
+    if (!out) return fail(VB_ERR_INVALID_ARG, "out is null");
+    *out = nullptr;
+    if (batch < 0) return fail(VB_ERR_INVALID_ARG, "batch < 0");
+    if (dt != VB_BF16 && dt != VB_F16) return fail(VB_ERR_UNSUPPORTED, "convolution plans are bf16/fp16 only");
+    if (batch > 0 && !desc) return fail(VB_ERR_INVALID_ARG, "null convolution descriptors");
+    std::vector<int32_t> M((size_t)batch), N((size_t)batch), K((size_t)batch), lda((size_t)batch),
+        ldb((size_t)batch), ldc((size_t)batch);
+    for (int i = 0; i < batch; ++i) {
+      const vb_conv_desc &c = desc[i];
+      if (c.nb < 1 || c.H < 1 || c.W < 1 || c.Cin < 1 || c.Cout < 1 || c.KH < 1 || c.KW < 1)
+        return fail(VB_ERR_INVALID_ARG, "conv %d: sizes must be >= 1", i);
+      if (c.KH != c.KW || c.KH > 8) return fail(VB_ERR_INVALID_ARG, "conv %d: square filters up to 8x8 only", i);
+      if (c.pad < 0 || c.pad >= c.KH) return fail(VB_ERR_INVALID_ARG, "conv %d: need 0 <= pad < KH", i);
+      const int64_t Ho = (int64_t)c.H + 2 * c.pad - c.KH + 1, Wo = (int64_t)c.W + 2 * c.pad - c.KW + 1;
+      if (Ho < 1 || Wo < 1) return fail(VB_ERR_INVALID_ARG, "conv %d: empty output", i);
+      if (c.ldb < c.Cout || c.ldc < c.Cout) return fail(VB_ERR_INVALID_ARG, "conv %d: ldb/ldc below Cout", i);
+      if (c.Cin % 8 || c.ldb % 8 || c.ldc % 8)
+        return fail(VB_ERR_ALIGNMENT, "conv %d: Cin, ldb and ldc must be multiples of 8 (16-byte rows)", i);
+      const int64_t m = (int64_t)c.nb * Ho * Wo, k = (int64_t)c.KH * c.KW * c.Cin;
+      if ((int64_t)c.nb * c.H * c.W * c.Cin >= ((int64_t)1 << 31) || m >= ((int64_t)1 << 31) || k >= (1 << 20))
+        return fail(VB_ERR_INVALID_ARG, "conv %d: too large", i);
+      M[(size_t)i] = (int32_t)m;
+      N[(size_t)i] = c.Cout;
+      K[(size_t)i] = (int32_t)k;
+      lda[(size_t)i] = (int32_t)k;     // unused by the im2col maps; satisfies lda >= K
+      ldb[(size_t)i] = c.ldb;
+      ldc[(size_t)i] = c.ldc;
     }
-    const TableDef *t = resolve_table(dt, tuning ? tuning->table_id : 0);
-    if (!t) return fail(VB_ERR_INVALID_ARG, "unknown table id %d", tuning ? tuning->table_id : -1);
-    if (device >= 0 && !table_runs_on(t, dt))
-      return fail(VB_ERR_UNSUPPORTED, "table %s has no kernel for this dtype", t->name);
-    const int64_t thr = (tuning && tuning->tlp_threshold > 0) ? tuning->tlp_threshold : t->tlp_threshold;
-    const int theta = (tuning && tuning->theta > 0) ? tuning->theta : t->theta;
-    vb_plan *p = new vb_plan();
-    p->device = device;
-    p->dt = dt;
-    p->batch = batch;
-    p->table = t;
-    p->policy = (int)policy;
-    p->tiling = tiling_engine(M, N, batch, *t, thr, pairs_allowed(M, N, K, batch, elem_bytes(dt)));
-    if (batch == 0) p->tiling.version_T = t->versions[0];
-    const std::vector<TileRec> all = enumerate_tiles(M, N, K, batch, p->tiling.row, *t);
-    if (all.size() > (size_t)INT32_MAX) {
-      delete p;
-      return fail(VB_ERR_INVALID_ARG, "more than 2^31 tiles");
-    }
-    // 2-SM pair tiles run in their own cluster kernel: batch them separately, pair blocks first.
-    std::vector<TileRec> tiles;
-    tiles.reserve(all.size());
-    for (const TileRec &r : all)
-      if (t->rows[p->tiling.row[r.gemm]].ctas == 2) tiles.push_back(r);
-    const size_t n_pair = tiles.size();
-    for (const TileRec &r : all)
-      if (t->rows[p->tiling.row[r.gemm]].ctas != 2) tiles.push_back(r);
-    Schedule sch;
-    sch.block_ptr.push_back(0);
-    for (int part = 0; part < 2; ++part) {
-      const std::vector<TileRec> sub(tiles.begin() + (part ? n_pair : 0), part ? tiles.end() : tiles.begin() + n_pair);
-      const Schedule sp = policy == VB_BATCH_THRESHOLD ? batch_threshold(sub, p->tiling.version_T, thr, theta)
-                          : policy == VB_BATCH_BINARY  ? batch_binary(sub, theta)
-                                                       : batch_none(sub);
-      const int32_t base = (int32_t)sch.slot_tile.size(), off = part ? (int32_t)n_pair : 0;
-      for (int32_t v : sp.slot_tile) sch.slot_tile.push_back(v + off);
-      for (size_t b = 1; b < sp.block_ptr.size(); ++b) sch.block_ptr.push_back(base + sp.block_ptr[b]);
-      if (part == 0) p->n_pair_blocks = (int)sch.block_ptr.size() - 1;
-    }
-    st = finish_plan(p, M, N, K, lda, ldb, ldc, tiles, sch);
-    if (st != VB_OK) {
-      delete p;
-      return st;
-    }
-    *out = p;
-    return VB_OK;
+    return plan_impl(device, dt, batch, M.data(), N.data(), K.data(), lda.data(), ldb.data(), ldc.data(), policy,
+                     tuning, desc, out);
   } catch (const std::bad_alloc &) {
     return fail(VB_ERR_OOM, "host allocation failed");
   } catch (...) {
@@ -586,12 +701,13 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
     const int n_pair = p->n_pair_blocks, n_single = n_blocks - n_pair;
     e = cudaSuccess;
     if (n_pair > 0) {
-      TcArgs a{p->d_block_ptr, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_pair, g_trace};
+      TcArgs a{p->d_block_ptr, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_pair, g_trace,
+               p->d_conv};
       e = launch_tc(a, 2 * std::min(n_pair, p->sm_count / 2), p->dt == VB_BF16, true, s);
     }
     if (e == cudaSuccess && n_single > 0) {
       TcArgs a{p->d_block_ptr + n_pair, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter + 2, n_single,
-               g_trace};
+               g_trace, p->d_conv};
       e = launch_tc(a, std::min(n_single, p->sm_count), p->dt == VB_BF16, false, s);
     }
   }

@@ -431,6 +431,18 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const uint8_t *mapA = maps + (a_tail ? MAP_A_TAIL : MAP_A) * 128;
         const int b_boxes = b_boxes_of((int)rank);
         const int ksteps_last = (ti.d.flags >> 8) & 7;
+        // implicit GEMM (vb_plan_conv): the window origin of this CTA's first output pixel
+        const bool conv = (ti.d.flags & kFlagConv) != 0;
+        ConvParam cv{};
+        int img = 0, oy = 0, ox = 0, ctap = 0, ccb = 0;
+        if (conv) {
+          cv = p.conv[ti.d.gemm];
+          const int hw = cv.Hout * cv.Wout;
+          img = row0 / hw;
+          const int rem = row0 - img * hw;
+          oy = rem / cv.Wout;
+          ox = rem - oy * cv.Wout;
+        }
         const int a_pages = BY * kBK * 2 / kPageBytes;
         const int need = a_pages + (Nh * kBK * 2 + kPageBytes - 1) / kPageBytes;
         for (int kb = 0; kb < ti.d.kblocks; ++kb, ++kbg) {
@@ -475,6 +487,17 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             if (i == 0 && a_box_rows == 0) continue;
             uint8_t *dst = i == 0 ? sa : sb + (i - 1) * kBK * geo.b_swz;
             const uint8_t *map = i == 0 ? mapA : mapB;
+            if (conv) {   // k-block kb = (tap ctap, channel block ccb)
+              if (i == 0) {
+                const int kh = ctap / cv.KW, kw = ctap - kh * cv.KW;
+                ptx::tma_load_im2col_4d(dst, map, &sh->full[slot], ccb * kBK, ox - cv.pad, oy - cv.pad, img,
+                                        (uint16_t)kw, (uint16_t)kh);
+              } else {
+                ptx::tma_load_2d(dst, map, &sh->full[slot], col0 + (i - 1) * (geo.b_swz / 2),
+                                 ctap * cv.Cin + ccb * kBK);
+              }
+              continue;
+            }
             const int c0 = i == 0 ? kb * kBK : col0 + (i - 1) * (geo.b_swz / 2);
             const int c1 = i == 0 ? row0 : kb * kBK;
             if (PAIR)
@@ -487,6 +510,10 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 #endif
           }
           VB_TADD(T_PROD_ISSUE);
+          if (conv && ++ccb == cv.ncb) {
+            ccb = 0;
+            ++ctap;
+          }
           advance(slot, sph, kSlots);
           if (pid == 0 && leader) sh->prod_kb = sh->prod_kb + 1u;
         }

@@ -64,6 +64,20 @@ constexpr int kMapsPerGemm = 6;
 enum MapIndex { MAP_A = 0, MAP_A_TAIL = 1, MAP_B = 2, MAP_B_TAIL = 3, MAP_C = 4, MAP_C_ST = 5 };
 static_assert(sizeof(TileDesc) == 32, "TileDesc must stay 32 bytes");
 
+// Implicit-GEMM convolution parameters per GEMM (vb_plan_conv).  A tile whose
+// TileDesc.flags has kFlagConv set loads A with TMA im2col copies: k-block kb covers filter tap
+// kb / ncb (tap = kh * KW + kw) and input channels [64 * (kb % ncb), +64); its B rows start at
+// tap * Cin + 64 * (kb % ncb).
+struct alignas(16) ConvParam {
+  int32_t Hout, Wout;   // output image size (pixels of one image = Hout * Wout)
+  int32_t Cin, KW;
+  int32_t pad;
+  int32_t ncb;          // channel blocks per tap: ceil(Cin / 64)
+  int32_t pad_[2];
+};
+static_assert(sizeof(ConvParam) == 32, "ConvParam must stay 32 bytes");
+constexpr uint16_t kFlagConv = 1u << 12;
+
 struct TcArgs {
   const int32_t *block_ptr;
   const TileDesc *tiles;    // [n_slots]
@@ -74,6 +88,7 @@ struct TcArgs {
   int32_t *counter;         // [0] dynamic work-list counter, [1] finished CTAs
   int32_t n_blocks;
   long long *trace;         // VB_TRACE builds only: per-role wait cycles (else nullptr)
+  const ConvParam *conv;    // [batch] for convolution plans (vb_plan_conv), else nullptr
 };
 
 // Tensor-core strategy geometry derived from a table row (BY, BX): TMA boxes and swizzles.

@@ -63,6 +63,16 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const void *tmap, uint64_
       "l"(tmap), "r"(c0), "r"(c1), "r"(smem_u32(bar))
       : "memory");
 }
+// im2col-mode TMA load over a 4-D NHWC map: coordinates {c, w, h, n} of the first window
+// origin, im2col offsets {w_off, h_off} (the filter tap) -- implicit-GEMM A tiles.
+__device__ __forceinline__ void tma_load_im2col_4d(void *dst, const void *tmap, uint64_t *bar, int32_t c, int32_t w,
+                                                   int32_t h, int32_t n, uint16_t w_off, uint16_t h_off) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], "
+      "[%6], {%7, %8};" ::"r"(smem_u32(dst)),
+      "l"(tmap), "r"(c), "r"(w), "r"(h), "r"(n), "r"(smem_u32(bar)), "h"(w_off), "h"(h_off)
+      : "memory");
+}
 // L2 cache policies for TMA (createpolicy): streamed data (C_old, C) is marked evict-first so
 // it does not push the reused A/B panels out of L2.
 __device__ __forceinline__ uint64_t policy_evict_first() {

@@ -20,7 +20,7 @@ from __future__ import annotations
 
 import numpy as np
 
-from .configs import (CONFIGS, googlenet_shapes, config_sizes, padded_ld,  # noqa: F401
+from .configs import (CONFIGS, googlenet_shapes, googlenet_convs, config_sizes, padded_ld,  # noqa: F401
                       elem_size, DTYPES)
 
 MASK64 = (1 << 64) - 1

@@ -63,6 +63,24 @@ def googlenet_shapes(nb: int = 1, first_stage_only: bool = False, module: str | 
     return out
 
 
+def googlenet_convs(nb: int = 1, first_stage_only: bool = False, module: str | None = None):
+    """The same inception-branch convolutions as dicts for the implicit-GEMM path (NEXT-3):
+    name, nb, H, W, Cin, Cout, KH, KW, pad (stride 1, "same" padding).  pool_proj is the 1x1
+    convolution applied to the (max-pooled) module input; the pooling itself is not part of
+    the GEMM path."""
+    out = []
+    for name, cin, hw, c1, r3, c3, r5, c5, pp in _INCEPTION:
+        if module is not None and name != module:
+            continue
+        branches = [("1x1", cin, c1, 1), ("3x3_reduce", cin, r3, 1), ("3x3", r3, c3, 3),
+                    ("5x5_reduce", cin, r5, 1), ("5x5", r5, c5, 5), ("pool_proj", cin, pp, 1)]
+        for bname, ci, co, k in branches:
+            if first_stage_only and bname in ("3x3", "5x5"):
+                continue
+            out.append(dict(name=f"{name}/{bname}", nb=nb, H=hw, W=hw, Cin=ci, Cout=co, KH=k, KW=k, pad=(k - 1) // 2))
+    return out
+
+
 CONFIGS = {
     "C1": dict(dtype="f32", desc="8 fp32 GEMMs, M/N/K uniform random in [16,128], seed 0", ab="random"),
     "C2": dict(dtype="f32", desc="256 fp32 GEMMs, M/N/K uniform random in [32,512]", ab="random"),
