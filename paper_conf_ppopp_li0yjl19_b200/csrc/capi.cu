@@ -412,6 +412,8 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
         const ConvParam &c = p->conv[ts.gemm];
         d.kblocks = g.K > 0 ? (g.K / c.Cin) * c.ncb : 0;
         d.flags |= kFlagConv;
+        const int last = c.Cin - 64 * (c.ncb - 1);   // channels in each tap's last block
+        if (last < 64) d.flags |= (uint16_t)(((last + 15) / 16) << 8);   // MMA K-steps of that block
       } else if (g.K % 64) {
         d.flags |= (uint16_t)(((g.K % 64 + 15) / 16) << 8);   // MMA K-steps of the last k-block
       }

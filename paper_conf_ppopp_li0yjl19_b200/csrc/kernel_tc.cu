@@ -467,7 +467,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           ++inflight;
           head = start + need;
           if (head == kPages) head = 0;
-          const bool k_tail = (kb == ti.d.kblocks - 1) && ksteps_last != 0;
+          const bool k_tail = !conv && (kb == ti.d.kblocks - 1) && ksteps_last != 0;   // conv: bits 8-10 mean per-tap steps
           const int b_rows = k_tail ? ksteps_last * 16 : kBK;
           const uint8_t *mapB = maps + (k_tail ? MAP_B_TAIL : MAP_B) * 128;
           uint8_t *sa = pages + (size_t)start * kPageBytes;
@@ -564,13 +564,21 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const uint64_t adesc0 = ptx::smem_desc(0, 16, 1024, 2);
         const uint64_t bdesc0 = ptx::smem_desc(0, kBK * geo.b_swz, 8 * geo.b_swz, blayout);
         const uint32_t b_step = (uint32_t)geo.b_swz;    // (16 * b_swz) >> 4
+        // implicit GEMM: the last channel block of every tap holds Cin % 64 channels; the K=16
+        // steps past them would multiply zero-filled A columns and are skipped
+        const bool conv = (ti.d.flags & kFlagConv) != 0;
+        const int ncb = conv ? p.conv[ti.d.gemm].ncb : 0;
+        int cb = 0;
         for (int kb = 0; kb < ti.d.kblocks; ++kb) {
           VB_TWAIT(T_MMA_FULL, ptx::mbar_wait(&sh->full[slot], sph));
           ptx::tc_fence_after();
           VB_T0();
           const uint32_t sa = ptx::smem_u32(pages + (size_t)sh->slot_page[slot] * kPageBytes);
           const uint32_t sb = sa + a_bytes;
-          const int ksteps = (kb == ti.d.kblocks - 1 && ((ti.d.flags >> 8) & 7)) ? ((ti.d.flags >> 8) & 7) : kBK / 16;
+          const int ksl = (ti.d.flags >> 8) & 7;
+          const int ksteps = conv ? ((cb == ncb - 1 && ksl) ? ksl : kBK / 16)
+                                  : ((kb == ti.d.kblocks - 1 && ksl) ? ksl : kBK / 16);
+          if (conv && ++cb == ncb) cb = 0;
           const uint64_t adesc = adesc0 | (uint64_t)(sa >> 4);
           const uint64_t bdesc = bdesc0 | (uint64_t)(sb >> 4);
           if (ptx::elect_lane0()) {

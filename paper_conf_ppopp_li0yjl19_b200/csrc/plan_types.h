@@ -67,7 +67,8 @@ static_assert(sizeof(TileDesc) == 32, "TileDesc must stay 32 bytes");
 // Implicit-GEMM convolution parameters per GEMM (vb_plan_conv).  A tile whose
 // TileDesc.flags has kFlagConv set loads A with TMA im2col copies: k-block kb covers filter tap
 // kb / ncb (tap = kh * KW + kw) and input channels [64 * (kb % ncb), +64); its B rows start at
-// tap * Cin + 64 * (kb % ncb).
+// tap * Cin + 64 * (kb % ncb).  Flags bits 8-10 then give the MMA K=16 steps of each tap's last
+// channel block (0 = 4).
 struct alignas(16) ConvParam {
   int32_t Hout, Wout;   // output image size (pixels of one image = Hout * Wout)
   int32_t Cin, KW;

@@ -18,10 +18,15 @@ ap.add_argument("--nb", type=int, default=1)
 ap.add_argument("--thr", type=int, default=0)
 ap.add_argument("--theta", type=int, default=0)
 args = ap.parse_args()
-info = vbinputs.CONFIGS[args.config]
-M, N, K = vbinputs.config_sizes(args.config, nb=args.nb)
-db = DeviceBatch(M, N, K, info["dtype"])
-db.fill(0, info["ab"])
+if args.config == "C3i":   # GoogleNet convolutions as implicit GEMMs (vb_plan_conv)
+    from paper_conf_ppopp_li0yjl19_b200.batch import ConvBatch
+    db = ConvBatch(vbinputs.googlenet_convs(nb=args.nb), "bf16")
+    db.fill(0, "conv")
+else:
+    info = vbinputs.CONFIGS[args.config]
+    M, N, K = vbinputs.config_sizes(args.config, nb=args.nb)
+    db = DeviceBatch(M, N, K, info["dtype"])
+    db.fill(0, info["ab"])
 plan = db.plan(vb.POLICIES[args.policy], tlp_threshold=args.thr, theta=args.theta)
 db.bind(plan)
 for _ in range(args.iters):
