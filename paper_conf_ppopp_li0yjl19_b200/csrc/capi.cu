@@ -23,7 +23,7 @@
 #include "tables.h"
 
 namespace vb {
-cudaError_t launch_f32(const F32Args &args, int n_blocks, int version_T, cudaStream_t stream);
+cudaError_t launch_f32(const F32Args &args, int grid, int version_T, bool slim, cudaStream_t stream);
 cudaError_t launch_f32_prep(uint8_t *tmaps, const void *const *A, const void *const *B, const GemmParam *gemms,
                             int batch, cudaStream_t stream);
 cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
@@ -232,7 +232,10 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
 #define VB_F32_CTAS_PER_SM 2
 #endif
   const int n_blocks = (int)p->block_ptr.size() - 1;
-  p->f32_grid = tc ? 0 : std::min(n_blocks, VB_F32_CTAS_PER_SM * p->sm_count);
+  // FFMA kernel residency: the B200 table's 128-thread variant runs four CTAs per SM, the
+  // 256-thread version (and the V100 profile) two
+  const bool slim = !tc && p->table->id == VB_TABLE_B200_FFMA && p->tiling.version_T == 128;
+  p->f32_grid = tc ? 0 : std::min(n_blocks, (slim ? 2 : 1) * VB_F32_CTAS_PER_SM * p->sm_count);
   const size_t o_or = off;
   if (!tc) off = align_up(off + (size_t)std::max(n_blocks, 1) * sizeof(int32_t), 256);
   const size_t o_ct = off;
@@ -697,7 +700,8 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
     F32Args a{p->d_block_ptr, p->d_slots, p->d_gemms, reinterpret_cast<const float *const *>(p->bound_A),
               reinterpret_cast<const float *const *>(p->bound_B), reinterpret_cast<float *const *>(p->bound_C),
               alpha, beta, p->d_order, p->d_tmaps, p->d_counter, n_blocks};
-    e = launch_f32(a, p->f32_grid, p->tiling.version_T, s);
+    e = launch_f32(a, p->f32_grid, p->tiling.version_T,
+                   p->table->id == VB_TABLE_B200_FFMA && p->tiling.version_T == 128, s);
   } else {
     // 2-SM pair tiles first (clusters of 2 over blocks [0, n_pair)), then the 1-SM tiles
     const int n_pair = p->n_pair_blocks, n_single = n_blocks - n_pair;

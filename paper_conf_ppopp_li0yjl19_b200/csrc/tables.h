@@ -46,13 +46,18 @@ struct TableDef {
 // V100 profile: the paper's constants (P255, P290).
 constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 128}, 65536, 256, 0, 0};
 
-// B200 FFMA profile (fp32): Table 2 shapes/sub-tiles (an FFMA design that still holds on
-// sm_100a), threshold re-set for 148 SMs (reading C-22).  Calibrated on B200: the 128-thread
-// version (16x8 sub-tiles, 255 registers, 8 warps per SM) is 13% slower than the 256-thread
-// version at two CTAs per SM on C2, so this profile offers the 256-thread version only.
-// Constants calibrated on B200 over the Fig. 8/9 grid + C1/C2 (scripts/calibrate_grid.py,
-// profiles/calibration_grid_f32_r01.json): TLP threshold 4 * 148 * 256, theta 64.
-constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 6, VB_TABLE2_ROWS, 1, {256, 0}, 4 * 148 * 256, 64, 0, 0};
+// B200 FFMA profile (fp32): Table 2's shapes with its 128-thread sub-tiles (an FFMA design that
+// still holds on sm_100a), threshold re-set for 148 SMs (reading C-22).  Calibrated on B200
+// (DESIGN.md §4, §6.2): the 128-thread version without the 128x128 row (16x8 sub-tiles need
+// 255 registers) runs four CTAs per SM -- one warp per SMSP per CTA, so the warps that share an
+// operand ring have equal scheduler priority -- and measured 6 % faster on C2 than the
+// 256-thread version at two CTAs per SM (0.312 vs 0.332 ms), which in turn beat the full
+// 128-thread version at one CTA per SM by 13 %.  TLP threshold 4 * 148 * 256 and theta 64 from
+// the grid calibration (scripts/calibrate_grid.py); C1/C2 are insensitive to them here.
+constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 5,
+                                     {{"small", 16, 16, 8, 1}, {"medium", 32, 32, 8, 1}, {"large", 64, 64, 8, 1},
+                                      {"tall", 128, 64, 8, 1}, {"wide", 64, 128, 8, 1}},
+                                     1, {128, 0}, 4 * 148 * 256, 64, 0, 0};
 
 // B200 tcgen05 profile (bf16/fp16): C tiles for tcgen05.mma with M in {64,128}; BK = 64 =
 // one 128-byte swizzled row of bf16; 256 threads per tile in Eq. 1.  Besides the paper's
