@@ -318,18 +318,26 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     // long-K tiles do not hoard blocks: the blocks in progress across the GPU stay a short
     // window of consecutive GEMMs and their A/B re-reads hit in L2.
     uint32_t t = 0, pushed_kb = 0;
-    int next = 0;
-    if (lane == 0) next = atomicAdd(p.counter, 1);
-    next = __shfl_sync(0xffffffffu, next, 0);
+    // the first block of every CTA (cluster) is static -- block = CTA (cluster) index -- so the
+    // first tile's descriptor read does not wait for an atomic round trip; later blocks are
+    // claimed from the counter, offset by the number of CTAs (clusters)
+    const int n_static = (int)gridDim.x / (PAIR ? 2 : 1);
+    // Software-pipelined by one block: while the tiles of block b are read and pushed, the
+    // CSR range of the next block (claimed one ahead) is already in flight and the block after
+    // it is being claimed, so each block costs one dependent global round trip, not three.
+    int b = (int)blockIdx.x / (PAIR ? 2 : 1);
+    int lim = (b < p.n_blocks && lane < 2) ? p.block_ptr[b + lane] : 0;
+    int nb = 0;
+    if (lane == 0) nb = n_static + atomicAdd(p.counter, 1);
+    nb = __shfl_sync(0xffffffffu, nb, 0);
     for (;;) {
-      const int b = next;
       if (b >= p.n_blocks) break;
+      int nb2 = nb;
       if (lane == 0) {
         VB_TWAIT(T_SCHED_BUDGET, while ((int)(pushed_kb - sh->prod_kb) > kKbAhead) __nanosleep(128));
-        next = atomicAdd(p.counter, 1);                 // claim one block ahead
+        if (nb < p.n_blocks) nb2 = n_static + atomicAdd(p.counter, 1);   // claim two ahead
       }
-      int lim = 0;
-      if (lane < 2) lim = p.block_ptr[b + lane];
+      const int lim_next = (nb < p.n_blocks && lane < 2) ? p.block_ptr[nb + lane] : 0;
       const int s0 = __shfl_sync(0xffffffffu, lim, 0), s1 = __shfl_sync(0xffffffffu, lim, 1);
       for (int base = s0; base < s1; base += 32) {
         const int n = min(32, s1 - base);
@@ -345,14 +353,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           }
           ptx::prefetch_tmap(maps + MAP_C * 128);
           if (d.N >= 8) ptx::prefetch_tmap(maps + MAP_C_ST * 128);
-          const float al = p.alpha[d.gemm], be = p.beta[d.gemm];
           const uint32_t tt = t + lane;
           const int e = (int)(tt % kRing);
           VB_TWAIT(T_SCHED_REMPTY, ptx::mbar_wait(&sh->rempty[e], ((tt / kRing) & 1u) ^ 1u));
           TileInfo &ti = sh->ring[e];
-          ti.d = d;
-          ti.alpha = al;
-          ti.beta = be;
+          ti.d = d;   // alpha / beta are read by their users (C producers, epilogue) off this chain
           if (PAIR) {                                 // mirror the entry into the peer's ring
             const uint32_t ra = ptx::mapa(&ti, 1);
             const uint4 *src = reinterpret_cast<const uint4 *>(&ti);
@@ -368,7 +373,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         pushed_kb += (uint32_t)kb;
         t += (uint32_t)n;
       }
-      next = __shfl_sync(0xffffffffu, next, 0);
+      b = nb;
+      lim = lim_next;
+      nb = __shfl_sync(0xffffffffu, nb2, 0);
     }
     if (lane == 0) {                                        // end marker
       const int e = (int)(t % kRing);
@@ -629,7 +636,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const TcGeom geo = tc_geom(BY, BX);
         const int row0 = ti.d.m0 + (int)rank * BY;
         const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C * 128;
-        const bool load = ti.beta != 0.f;
+        const bool load = p.beta[ti.d.gemm] != 0.f;
         const int nch = live_chunks(geo, ti.d.N, ti.d.n0);
         for (int ch = 0; ch < nch; ++ch) {
           VB_TWAIT(T_CPROD_CEMPTY, ptx::mbar_wait(&sh->cempty[cs], cph ^ 1u));
@@ -677,6 +684,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       if (lane == 0) ring_release(re);
       advance(re, rph, kRing);
       if (ti.d.gemm < 0) break;
+      const float t_alpha = p.alpha[ti.d.gemm], t_beta = p.beta[ti.d.gemm];   // used after the accumulator wait
       const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
       const TcGeom geo = tc_geom(BY, BX);
       const int row0 = ti.d.m0 + (int)rank * BY;     // this CTA's first row of the tile
@@ -735,9 +743,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           if (row_ok && live) {
 #endif
             if (hcols == 32)
-              epi_row<AB_FMT, 4>(cb, row, geo.c_swz, half * 4, acc, ti.alpha, ti.beta);
+              epi_row<AB_FMT, 4>(cb, row, geo.c_swz, half * 4, acc, t_alpha, t_beta);
             else
-              epi_row<AB_FMT, 2>(cb, row, geo.c_swz, half * 2, acc, ti.alpha, ti.beta);
+              epi_row<AB_FMT, 2>(cb, row, geo.c_swz, half * 2, acc, t_alpha, t_beta);
           }
           VB_TADD(T_EPI_MATH);
         }
