@@ -87,6 +87,23 @@ struct TileInfo {          // one tile ring entry (48 bytes)
   int32_t pad[2];
 };
 static_assert(sizeof(TileInfo) == 48, "TileInfo size");
+// Opt-in timeline (build with -DVB_TIMELINE, measurement only): the first %globaltimer stamp
+// of each event of CTA 0 into p.trace[i] (zeroed by the caller).  Events: 0 entry, 1 setup
+// done, 2 first ring entry pushed, 3 first k-block armed by a producer, 4 MMA saw its first
+// k-block, 5 first accumulator committed, 6 epilogue saw it, 7 epilogue done with it, 8 its
+// stores complete, 9 teardown barrier passed, 10 exit.
+#ifdef VB_TIMELINE
+__device__ __forceinline__ void vb_stamp(long long *buf, int i) {
+  if (blockIdx.x == 0 && buf) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    atomicCAS(reinterpret_cast<unsigned long long *>(buf) + i, 0ull, t);
+  }
+}
+#define VB_STAMP(i) vb_stamp(p.trace, i)
+#else
+#define VB_STAMP(i)
+#endif
 
 struct Shared {
   uint64_t full[kSlots], empty[kSlots];
@@ -250,6 +267,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   // 1024-byte aligned (SW128 atoms); offsetting smem_raw itself keeps the shared address space
   // visible to the compiler, so C-slot and barrier accesses compile to LDS/STS, not generic LD/ST.
   uint8_t *smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
+  if (threadIdx.x == 0) VB_STAMP(0);
   uint8_t *pages = smem;
   uint8_t *cbuf = smem + (size_t)kPages * kPageBytes;
   Shared *sh = reinterpret_cast<Shared *>(cbuf + (size_t)kCSlots * kCSlotBytes);
@@ -304,6 +322,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = sh->tmem_base;
+  if (threadIdx.x == 0) VB_STAMP(1);
   const uint8_t *tmaps = reinterpret_cast<const uint8_t *>(p.tmaps);
 #ifdef VB_TRACE
   long long tr[kTraceSlots];
@@ -367,6 +386,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             ptx::mbar_arrive_remote(ptx::mapa(&sh->rfull[e], 1));
           }
           ptx::mbar_arrive(&sh->rfull[e]);
+          VB_STAMP(2);
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) kb += __shfl_xor_sync(0xffffffffu, kb, o);
@@ -486,6 +506,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
               uint32_t bytes = (uint32_t)(a_box_rows_of(0) * kBK * 2 + b_boxes_of(0) * b_rows * geo.b_swz);
               if (PAIR) bytes += (uint32_t)(a_box_rows_of(1) * kBK * 2 + b_boxes_of(1) * b_rows * geo.b_swz);
               ptx::mbar_arrive_expect_tx(&sh->full[slot], bytes);
+              VB_STAMP(3);
             }
           }
           // box 0 = A, boxes 1..b_boxes = B; box i goes to producer (i + kbg) % kProducers
@@ -578,6 +599,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         int cb = 0;
         for (int kb = 0; kb < ti.d.kblocks; ++kb) {
           VB_TWAIT(T_MMA_FULL, ptx::mbar_wait(&sh->full[slot], sph));
+          VB_STAMP(4);
           ptx::tc_fence_after();
           VB_T0();
           const uint32_t sa = ptx::smem_u32(pages + (size_t)sh->slot_page[slot] * kPageBytes);
@@ -614,6 +636,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             ptx::mma_commit_pair(&sh->tfull[e]);
           else
             ptx::mma_commit(&sh->tfull[e]);         // accumulator ready for the epilogue
+          VB_STAMP(5);
         }
       }
     }
@@ -709,6 +732,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       tr[T_EPI_HEAD] += clock64() - _head_t0;
 #endif
       VB_TWAIT(T_EPI_TFULL, ptx::mbar_wait(&sh->tfull[e], aph));
+      if (lane == 0) VB_STAMP(6);
       ptx::tc_fence_after();
 #ifdef VB_TRACE
       const long long _tile_t0 = clock64();
@@ -808,8 +832,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 #ifdef VB_TRACE
       tr[T_EPI_LOOP] += clock64() - _tile_t0;
 #endif
+      if (lane == 0) VB_STAMP(7);
     }
-    if (storer && lane == 0) ptx::bulk_wait0();
+    if (storer && lane == 0) {
+      ptx::bulk_wait0();
+      VB_STAMP(8);
+    }
   }
 #ifdef VB_TRACE
   tr[T_TOTAL] = clock64() - t_start;
@@ -824,6 +852,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   else
     __syncthreads();
   ptx::tc_fence_after();
+  if (threadIdx.x == 0) VB_STAMP(9);
   if (warp == 1) {
     if (PAIR)
       ptx::tmem_dealloc_pair(tmem_base, kTmemCols);
@@ -839,6 +868,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       atomicExch(&p.counter[1], 0);
       __threadfence();
     }
+    VB_STAMP(10);
   }
 }
 

@@ -39,7 +39,10 @@ bool pairs_allowed(const int32_t *M, const int32_t *N, const int32_t *K, int bat
     if (M[i] > 0 && N[i] > 0)
       bytes += (__int128)elem_bytes * ((int64_t)M[i] * K[i] + (int64_t)K[i] * N[i]) + (__int128)2 * elem_bytes * M[i] * N[i];
   }
-  return bytes > 0 && flops >= (__int128)128 * bytes;
+#ifndef VB_PAIR_MIN_AI
+#define VB_PAIR_MIN_AI 128
+#endif
+  return bytes > 0 && flops >= (__int128)VB_PAIR_MIN_AI * bytes;
 }
 
 TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const TableDef &t,

@@ -94,3 +94,15 @@ def test_invalid_descriptors_rejected():
             vb.plan_conv([bad], "bf16")
     with pytest.raises(vb.VbError):
         vb.plan_conv([good], "f32")
+
+
+def test_googlenet_nb32_sampled_convs():
+    # the bench's C3i size at nb = 32 (every branch, 25 088 output pixels per conv); the oracle
+    # checks a sample of the convolutions (largest K, a 5x5, a 1x1, the first and the last)
+    convs = vbinputs.googlenet_convs(nb=32)
+    db, _ = _run(convs, "bf16")
+    ks = [c["KH"] * c["KW"] * c["Cin"] for c in convs]
+    pick = sorted({0, len(convs) - 1, int(np.argmax(ks)),
+                   next(i for i, c in enumerate(convs) if c["KH"] == 5),
+                   next(i for i, c in enumerate(convs) if c["KH"] == 1 and c["Cin"] > 500)})
+    check_convs(db, pick, SEED, "conv")
