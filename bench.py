@@ -435,9 +435,14 @@ def main_ours(args):
     if not torch.cuda.is_available():
         print(json.dumps({"metric": METRIC, "error": "no CUDA device"}))
         return 1
+    # VB_BENCH_SHARE_GPU=1 (testing the N > 1 code path on a one-GPU box only): every rank uses
+    # cuda:0 and the gloo backend for the barrier and the timing gathers
+    share = os.environ.get("VB_BENCH_SHARE_GPU") == "1"
+    if share:
+        local = 0
     torch.cuda.set_device(local)
-    dist_init(world, "nccl")
-    dist_device = torch.device("cuda", local)
+    dist_init(world, "gloo" if share else "nccl")
+    dist_device = torch.device("cpu") if share else torch.device("cuda", local)
     peaks = load_peaks()
     res, db, plan = run_config(args.config, args, world, rank, local, peaks, dist_device, headline=True)
     aux = {}
