@@ -235,7 +235,10 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
   // FFMA kernel residency: the B200 table's 128-thread variant runs four CTAs per SM, the
   // 256-thread version (and the V100 profile) two
   const bool slim = !tc && p->table->id == VB_TABLE_B200_FFMA && p->tiling.version_T == 128;
-  p->f32_grid = tc ? 0 : std::min(n_blocks, (slim ? 2 : 1) * VB_F32_CTAS_PER_SM * p->sm_count);
+#ifndef VB_F32_SLIM_CTAS
+#define VB_F32_SLIM_CTAS 4
+#endif
+  p->f32_grid = tc ? 0 : std::min(n_blocks, (slim ? VB_F32_SLIM_CTAS : VB_F32_CTAS_PER_SM) * p->sm_count);
   const size_t o_or = off;
   if (!tc) off = align_up(off + (size_t)std::max(n_blocks, 1) * sizeof(int32_t), 256);
   const size_t o_ct = off;
