@@ -277,11 +277,12 @@ def pairs_allowed(Ms, Ns, Ks, es: int = 2) -> bool:
 
 
 def plan(Ms, Ns, Ks, table: Table, policy: int = POLICY_THRESHOLD,
-         tlp_threshold: int | None = None, theta: int | None = None, es: int = 2) -> Plan:
+         tlp_threshold: int | None = None, theta: int | None = None, es: int = 2, allow_pairs: bool = True) -> Plan:
+    """allow_pairs=False: 1-SM strategies only (the implicit-GEMM convolution plans)."""
     thr = table.tlp_threshold if tlp_threshold is None else tlp_threshold
     th = table.theta if theta is None else theta
     Ms = [int(v) for v in Ms]; Ns = [int(v) for v in Ns]; Ks = [int(v) for v in Ks]
-    tr = tiling_engine(Ms, Ns, table, thr, pairs_allowed(Ms, Ns, Ks, es))
+    tr = tiling_engine(Ms, Ns, table, thr, allow_pairs and pairs_allowed(Ms, Ns, Ks, es))
     all_tiles = enumerate_tiles(Ms, Ns, Ks, tr.rows, table)
     # 2-SM pair tiles run in their own (cluster) kernel: the batching engine packs the pair
     # tiles and the single tiles separately (each keeps enumeration order); pair blocks first.

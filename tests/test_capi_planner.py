@@ -141,3 +141,32 @@ def test_random_plans_match_oracle(sz, tid, policy, thr, theta):
 def test_lpt_matches_oracle(sz, ranks):
     M = [s[0] for s in sz]; N = [s[1] for s in sz]; K = [s[2] for s in sz]
     assert list(nv.shard_lpt(M, N, K, ranks)) == pr.shard_lpt(M, N, K, ranks)
+
+
+@pytest.mark.parametrize("nb", [1, 4, 32])
+@pytest.mark.parametrize("policy", [vb.VB_BATCH_THRESHOLD, vb.VB_BATCH_BINARY])
+def test_conv_plan_is_the_oracle_plan_of_its_gemm_view(nb, policy):
+    # vb_plan_conv plans the GEMM view M = nb*Hout*Wout, N = Cout, K = KH*KW*Cin with 1-SM strategies
+    convs = vbinputs.googlenet_convs(nb=nb)
+    descs = [dict(c, ldb=int(vbinputs.padded_ld(c["Cout"], "bf16")), ldc=int(vbinputs.padded_ld(c["Cout"], "bf16")))
+             for c in convs]
+    plan = nv.plan_conv(descs, "bf16", policy, device=-1)
+    M = [c["nb"] * c["H"] * c["W"] for c in convs]
+    N = [c["Cout"] for c in convs]
+    K = [c["KH"] * c["KW"] * c["Cin"] for c in convs]
+    ref = pr.plan(M, N, K, pr.B200_TC, policy, allow_pairs=False)
+    _assert_same(plan, ref)
+    assert all(pr.B200_TC.rows[r].ctas == 1 for r in ref.tiling.rows)
+
+
+def test_conv_plan_validation_on_host():
+    good = dict(nb=2, H=8, W=8, Cin=16, Cout=24, KH=3, KW=3, pad=1, ldb=24, ldc=32)
+    assert nv.plan_conv([good], "bf16", device=-1).info()["n_tiles"] >= 1
+    bad_cases = [dict(good, Cin=12), dict(good, KW=5), dict(good, pad=3), dict(good, ldc=16),
+                 dict(good, KH=9, KW=9), dict(good, nb=0), dict(good, H=1, W=1, pad=0), dict(good, ldb=20)]
+    for bad in bad_cases:
+        with pytest.raises(vb.VbError):
+            nv.plan_conv([bad], "bf16", device=-1)
+    with pytest.raises(vb.VbError):
+        nv.plan_conv([good], "f32", device=-1)
+    assert nv.plan_conv([], "bf16", device=-1).info()["n_tiles"] == 0
