@@ -3,16 +3,17 @@
 // tensor-core MMA accumulating in TMEM.
 //
 // One CTA per SM (grid = min(Block_NUM, #SMs)), 16 warps:
-//   warp 0      scheduler: claims the next block (work list) with an atomic (one block
-//               ahead), loads its tile descriptors (one 32-byte record per tile, lanes in
-//               parallel) and alpha/beta into a 32-entry smem tile ring, prefetches the tiles'
-//               tensor maps; lookahead is bounded in k-blocks so the GPU works on a short
-//               window of GEMMs at a time (L2 reuse of A/B).
+//   warp 0      scheduler: starts with block = CTA index, then claims blocks (work lists)
+//               with an atomic, software-pipelined one block ahead; loads their tile
+//               descriptors (one 32-byte record per tile, lanes in parallel) into a 32-entry
+//               smem tile ring and prefetches the tiles' tensor maps; lookahead is bounded in
+//               k-blocks so the GPU works on a short window of GEMMs at a time (L2 reuse of A/B).
 //   warp 1      TMEM owner + MMA issuer: one thread issues tcgen05.mma (M = BY, N = BX,
 //               K = 16) into an accumulator ring of 512 TMEM columns (up to 8 tiles in flight).
 //   warps 2-3   C_old producers: TMA-load C_old chunks (BY x 64) per epilogue quarter into a
 //               4-slot ring when beta != 0 (C is never read when beta == 0, reading C-16).
-//   warps 4-7   A/B producers: stream each tile's k-blocks (A: BY x 64, B: 64 x BX) with TMA
+//   warps 4-7   A/B producers: stream each tile's k-blocks (A: BY x 64, B: 64 x BX; for an
+//               implicit-GEMM convolution tile A comes from TMA im2col copies) with TMA
 //               into a PAGED ring (18 pages of 8 KB; a k-block takes 2 pages for 64x32 ... 6
 //               for 128x256, so small tiles keep up to 9 k-blocks in flight — the paper's ILP
 //               concern for small K, P151/P259, as TMA depth).  One thread issues only ~1 TMA
@@ -81,10 +82,9 @@ constexpr int kAcc = 8;                    // accumulators in flight (ring entri
 constexpr int kEpiWarps = 8;               // two per TMEM lane quarter, splitting each chunk's columns
 constexpr uint32_t kRingConsumers = kProducers + 1 + kCProducers + kEpiWarps;
 
-struct TileInfo {          // one tile ring entry (48 bytes)
+struct TileInfo {          // one tile ring entry (48 bytes: three 16-byte DSMEM stores in a pair)
   TileDesc d;
-  float alpha, beta;
-  int32_t pad[2];
+  int32_t pad[4];
 };
 static_assert(sizeof(TileInfo) == 48, "TileInfo size");
 // Opt-in timeline (build with -DVB_TIMELINE, measurement only): the first %globaltimer stamp
