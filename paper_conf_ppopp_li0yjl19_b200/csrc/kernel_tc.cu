@@ -72,6 +72,7 @@ constexpr int kNGran = VB_NGRAN;          // MMA N granularity per CTA for edge 
 constexpr int kPages = VB_PAGES;           // 144 KB of A/B staging (default)
 constexpr int kSlots = 16;                 // k-blocks in flight (bounded by pages anyway)
 constexpr int kCSlots = VB_CSLOTS;
+static_assert(kCSlots >= 2, "the epilogue defers each store's completion by one chunk: one C slot deadlocks");
 constexpr int kCSlotBytes = 128 * 128;     // BY rows x 128 B
 constexpr int kRing = 32;                  // tile-descriptor ring entries
 constexpr int kKbAhead = VB_KBAHEAD;       // scheduler lookahead budget in k-blocks (L2 locality)
