@@ -322,6 +322,31 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
         f"inputs ({db.arena_bytes() / 1e9:.1f} GB per rank) >> L2 (126 MB); no flush",
         "launches": pinfo["launches_per_exec"] * steps, "clocks": clk, "batch_rank": int(db.batch),
     }
+    if not headline and small and world == 1:
+        # the small configs also with the step (bind + exec) captured in one CUDA
+        # graph and replayed (launch overhead amortised), L2 flushed outside the graph
+        g_stream = torch.cuda.Stream(dev)
+        graph = torch.cuda.CUDAGraph()
+        g_stream.wait_stream(stream)
+        with torch.cuda.stream(g_stream):
+            step()
+            torch.cuda.synchronize(dev)
+            with torch.cuda.graph(graph, stream=g_stream):
+                db.bind(plan, g_stream)
+                db.run_bound(plan, g_stream)
+        torch.cuda.synchronize(dev)
+        gts = []
+        for _ in range(steps):
+            flush.fill_(1)
+            s0 = torch.cuda.Event(enable_timing=True)
+            e0 = torch.cuda.Event(enable_timing=True)
+            s0.record(stream)
+            graph.replay()
+            e0.record(torch.cuda.current_stream(dev))
+            torch.cuda.synchronize(dev)
+            gts.append(s0.elapsed_time(e0))
+        res["graph_step_ms"] = float(np.median(gts))
+        del graph
     if headline and args.e2e_steps > 0:
         res["e2e"] = run_e2e(db, plan, args, world, dist_device, flops_all, stream, dev)
     del flush
@@ -457,6 +482,8 @@ def main_ours(args):
                         "plan_ms": round(r["plan_ms"], 2), "roofline": _round(r["roofline"]),
                         "n_tiles": r["plan"]["n_tiles"], "n_blocks": r["plan"]["n_blocks"], "l2": r["l2"],
                         "policy": r["policy_chosen"]}
+            if "graph_step_ms" in r:
+                aux[cfg]["cuda_graph_step_ms"] = round(r["graph_step_ms"], 4)
             del d2, p2
             torch.cuda.empty_cache()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -85,9 +85,7 @@ struct vb_plan {
   std::vector<ConvParam> conv;      // convolution plans (vb_plan_conv): one per GEMM, else empty
   std::vector<vb_conv_desc> conv_desc;
   ConvParam *d_conv = nullptr;
-  int32_t *d_counter = nullptr;     // work-list counters: pair (FFMA) kernel [0], [1] and 1-SM kernel
-                                    // [2], [3], one per launch parity (double-buffered)
-  uint32_t epoch = 0;               // launches since the last bind
+  int32_t *d_counter = nullptr;     // pair (FFMA) kernel [0] work-list, [1] finished CTAs; 1-SM kernel [2], [3]
   int n_pair_blocks = 0;            // blocks [0, n_pair_blocks) hold 2-SM pair tiles
   int sm_count = 0;
   const void *const *bound_A = nullptr;   // last vb_plan_bind
@@ -682,12 +680,10 @@ extern "C" vb_status vb_plan_bind(vb_plan_t p, const void *const *A, const void 
   DeviceGuard g(p->device);
   if (g.err != cudaSuccess) return cuda_fail(g.err, "cudaSetDevice");
   if (p->dt == VB_F32) {
-    p->epoch = 0;
     cudaError_t e = launch_f32_prep(p->d_tmaps, A, B, p->d_gemms, p->batch, p->d_counter,
                                     static_cast<cudaStream_t>(stream));
     return e == cudaSuccess ? VB_OK : cuda_fail(e, "prep kernel launch");
   }
-  p->epoch = 0;
   cudaError_t e = launch_tc_prep(p->d_tmaps, A, B, C, p->d_gemms, p->batch, p->d_counter,
                                  static_cast<cudaStream_t>(stream));
   return e == cudaSuccess ? VB_OK : cuda_fail(e, "prep kernel launch");
@@ -703,13 +699,11 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
   if (g.err != cudaSuccess) return cuda_fail(g.err, "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   const int n_blocks = (int)p->block_ptr.size() - 1;
-  const int cur = (int)(p->epoch & 1u), nxt = cur ^ 1;   // this launch's / the next launch's counters
-  ++p->epoch;
   cudaError_t e;
   if (p->dt == VB_F32) {
     F32Args a{p->d_block_ptr, p->d_slots, p->d_gemms, reinterpret_cast<const float *const *>(p->bound_A),
               reinterpret_cast<const float *const *>(p->bound_B), reinterpret_cast<float *const *>(p->bound_C),
-              alpha, beta, p->d_order, p->d_tmaps, p->d_counter + cur, p->d_counter + nxt, n_blocks};
+              alpha, beta, p->d_order, p->d_tmaps, p->d_counter, n_blocks};
     e = launch_f32(a, p->f32_grid, p->tiling.version_T,
                    p->table->id == VB_TABLE_B200_FFMA && p->tiling.version_T == 128, s);
   } else {
@@ -717,13 +711,13 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
     const int n_pair = p->n_pair_blocks, n_single = n_blocks - n_pair;
     e = cudaSuccess;
     if (n_pair > 0) {
-      TcArgs a{p->d_block_ptr, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter + cur,
-               p->d_counter + nxt, n_pair, g_trace, p->d_conv};
+      TcArgs a{p->d_block_ptr, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_pair, g_trace,
+               p->d_conv};
       e = launch_tc(a, 2 * std::min(n_pair, p->sm_count / 2), p->dt == VB_BF16, true, s);
     }
     if (e == cudaSuccess && n_single > 0) {
-      TcArgs a{p->d_block_ptr + n_pair, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter + 2 + cur,
-               p->d_counter + 2 + nxt, n_single, g_trace, p->d_conv};
+      TcArgs a{p->d_block_ptr + n_pair, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter + 2, n_single,
+               g_trace, p->d_conv};
       e = launch_tc(a, std::min(n_single, p->sm_count), p->dt == VB_BF16, false, s);
     }
   }

@@ -291,11 +291,6 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   };
 
   if (threadIdx.x == 0) {
-    // work-list counters are double-buffered across launches of a plan: this launch claims from
-    // p.counter (zeroed by the previous launch or by bind) and zeroes the next launch's, which
-    // the previous launch -- complete in stream order -- was the last to use.  No CTA has to
-    // detect that it finished last.
-    if (blockIdx.x == 0) *p.counter_next = 0;
     for (int i = 0; i < kSlots; ++i) {
       ptx::mbar_init(&sh->full[i], 1);
       ptx::mbar_init(&sh->empty[i], 1);
@@ -865,7 +860,18 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     else
       ptx::tmem_dealloc(tmem_base, kTmemCols);
   }
-  if (threadIdx.x == 0) VB_STAMP(10);
+  // The last CTA to finish resets the work-list counter, so back-to-back launches of the same
+  // bound plan -- including replays of a CUDA graph that captured only vb_exec_bound -- need no
+  // reset.  Every CTA made its final claim (one that returned >= n_blocks) before getting here.
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(&p.counter[1], 1) == (int)gridDim.x - 1) {
+      atomicExch(&p.counter[0], 0);
+      atomicExch(&p.counter[1], 0);
+      __threadfence();
+    }
+    VB_STAMP(10);
+  }
 }
 
 // Bind-time prep: patch the global address of every per-GEMM tensor map (A, B, C) with the
@@ -878,7 +884,7 @@ __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
                            const GemmParam *gemms, int batch, int32_t *counter) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i == 0) {
-    counter[0] = counter[1] = 0;   // pair kernel (two launch parities)
+    counter[0] = counter[1] = 0;   // pair kernel
     counter[2] = counter[3] = 0;   // 1-SM kernel
   }
   if (i >= batch * kMapsPerGemm) return;

@@ -36,8 +36,7 @@ struct F32Args {
   const float *beta;
   const int32_t *order;   // claim order of the blocks, heaviest first (execution detail, not part of the plan)
   const void *tmaps;      // CUtensorMap[batch][kF32MapsPerGemm] (A, B), 128-byte aligned
-  int32_t *counter;       // this launch's work-list counter (zero at launch)
-  int32_t *counter_next;  // the next launch's counter: zeroed by this launch (double buffering)
+  int32_t *counter;       // [0] work-list counter, [1] finished CTAs (reset by the last CTA to finish)
   int32_t n_blocks;
 };
 // fp32 tensor maps per GEMM: A (box 32 x BY, 128-byte swizzle) and B (box min(BX,32) x 32).
@@ -87,8 +86,7 @@ struct TcArgs {
   void *const *C;           // C pointers (direct stores of row tails that TMA cannot clip)
   const float *alpha;
   const float *beta;
-  int32_t *counter;         // this launch's work-list counter (zero at launch)
-  int32_t *counter_next;    // the next launch's counter: zeroed by this launch (double buffering)
+  int32_t *counter;         // [0] work-list counter, [1] finished CTAs (reset by the last CTA to finish)
   int32_t n_blocks;
   long long *trace;         // VB_TRACE builds only: per-role wait cycles (else nullptr)
   const ConvParam *conv;    // [batch] for convolution plans (vb_plan_conv), else nullptr

@@ -319,3 +319,39 @@ def test_plan_tune_keeps_faster_and_is_exact(dtype):
     db.run(plan)
     torch.cuda.synchronize()
     check_batch(db, range(db.batch), SEED, "random")
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_cuda_graph_replays_of_exec_bound(dtype):
+    # vb_exec_bound captured alone in a CUDA graph: every replay must claim all work lists again
+    # (the kernels reset their work-list counter themselves), and give the same exact result
+    M, N, K = vbinputs.config_sizes("C2")
+    M, N, K = M[:48], N[:48], K[:48]
+    db = DeviceBatch(M, N, K, dtype)
+    db.fill(SEED)
+    plan = db.plan()
+    c0 = db.C.clone()
+    db.bind(plan)
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(s):
+        db.run_bound(plan, s)                 # warm-up outside the capture
+        torch.cuda.synchronize()
+        db.C.copy_(c0)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=s):
+            db.run_bound(plan, s)
+    torch.cuda.synchronize()
+    first = None
+    for rep in range(4):
+        db.C.copy_(c0)
+        torch.cuda.synchronize()
+        g.replay()
+        torch.cuda.synchronize()
+        got = [db.c(g).clone() for g in range(len(M))]   # the matrices (arena padding is undefined)
+        if first is None:
+            first = got
+            check_batch(db, range(len(M)), SEED, "random")
+        else:
+            assert all(torch.equal(a, b) for a, b in zip(first, got)), f"replay {rep} differs"
