@@ -80,7 +80,7 @@ if __name__ == "__main__":
     tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
     os.makedirs(PROF, exist_ok=True)
     res = {}
-    for cfg in ("C5", "C4", "C2", "C3i"):
+    for cfg in ("C5", "C4", "C2", "C3", "C3i"):
         p = os.path.join(OUT, f"prof_{cfg}.ncu-rep")
         if os.path.exists(p):
             res[cfg] = summarize(p)
