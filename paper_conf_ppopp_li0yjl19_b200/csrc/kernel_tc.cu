@@ -53,6 +53,9 @@ constexpr int kPageBytes = 8192;
 #ifndef VB_KBAHEAD
 #define VB_KBAHEAD 8
 #endif
+#ifndef VB_KB_PREFETCH
+#define VB_KB_PREFETCH 0   // experiment: L2 prefetch of each A/B box this many k-blocks ahead
+#endif
 // L2 evict-first hints on the C_old loads / C stores.  Measured off by default: with the load
 // hint, C5 read 1.3x its compulsory DRAM bytes (a 500^3 batch: C_old fetched ~1.6x) and ran
 // 6% slower; without it DRAM reads are within 1-2% of the compulsory bytes.
@@ -536,6 +539,16 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
               ptx::tma_load_2d_hint(dst, map, &sh->full[slot], c0, c1, ab_policy);
 #else
               ptx::tma_load_2d(dst, map, &sh->full[slot], c0, c1);
+#endif
+#if VB_KB_PREFETCH > 0
+            // start the DRAM fetch of the same box VB_KB_PREFETCH k-blocks ahead into L2
+            if (kb + VB_KB_PREFETCH < ti.d.kblocks) {
+              const uint8_t *pmap = i == 0 ? mapA : maps + MAP_B * 128;
+              if (i == 0)
+                ptx::tma_prefetch_2d(pmap, (kb + VB_KB_PREFETCH) * kBK, row0);
+              else
+                ptx::tma_prefetch_2d(pmap, c0, (kb + VB_KB_PREFETCH) * kBK);
+            }
 #endif
           }
           VB_TADD(T_PROD_ISSUE);
