@@ -391,12 +391,14 @@ def run_e2e(db, plan, args, world, dist_device, flops_all, stream, dev):
             hi = int(off[g1]) if g1 < db.batch else arena.numel()
             rng[name] = (lo, hi)
         chunks.append((g0, g1, sub, rng))
-    s_h2d = torch.cuda.Stream(dev)
+    n_up = max(1, int(os.environ.get("VB_E2E_UPLOAD_STREAMS", "1")))
+    s_up = [torch.cuda.Stream(dev) for _ in range(n_up)]   # uploads alternate between these
     s_d2h = torch.cuda.Stream(dev)
 
     def step():
         prev_d2h = []
-        for g0, g1, sub, rng in chunks:
+        for ci, (g0, g1, sub, rng) in enumerate(chunks):
+            s_h2d = s_up[ci % n_up]
             with torch.cuda.stream(s_h2d):
                 for name, dst, src in (("A", db.A, hA), ("B", db.B, hB), ("C", db.C, hC)):
                     lo, hi = rng[name]
@@ -429,10 +431,12 @@ def run_e2e(db, plan, args, world, dist_device, flops_all, stream, dev):
     s = torch.cuda.Event(enable_timing=True)
     e = torch.cuda.Event(enable_timing=True)
     s.record(stream)
-    s_h2d.wait_stream(stream)
+    for su in s_up:
+        su.wait_stream(stream)
     for _ in range(args.e2e_steps):
         step()
-        s_h2d.wait_stream(stream)                    # next step's uploads after this step's results
+        for su in s_up:
+            su.wait_stream(stream)                   # next step's uploads after this step's results
     e.record(stream)
     torch.cuda.synchronize(dev)
     ms = s.elapsed_time(e) / args.e2e_steps
