@@ -159,8 +159,10 @@ vb_status vb_plan_conv(int device, vb_dtype dt, int32_t batch, const vb_conv_des
  *  C        DEVICE array  [batch] of DEVICE pointers (16-byte aligned), read+written.
  *  alpha, beta  DEVICE fp32 arrays [batch].
  *  stream   cudaStream_t as void*.
- * Never allocates, never synchronises.  Enqueues at most two kernels (a descriptor
- * prep kernel, then the GEMM kernel; the fp32 path needs no prep kernel).  The caller
+ * Never allocates, never synchronises.  Enqueues at most three kernels: the descriptor
+ * prep kernel (tensor-map address patch and work-counter reset), then the GEMM kernel(s) --
+ * fp32: one FFMA kernel; bf16/fp16: the 2-SM pair kernel (if the plan has pair tiles) and
+ * the 1-SM kernel.  All of it may be captured in a CUDA graph.  The caller
  * keeps every buffer alive until the stream work completes.  A plan may be re-executed
  * with new pointers / alpha / beta, but not concurrently on two streams.
  * Returns VB_ERR_CUDA if a launch fails (vb_last_error() has the CUDA message).
@@ -174,8 +176,10 @@ vb_status vb_exec_vbatched(vb_plan_t plan, const void *const *A, const void *con
  *  vb_plan_bind   records the DEVICE pointer arrays A, B, C in the plan and enqueues the
  *                 descriptor prep kernel (tensor-map address patch) on `stream`.  The arrays
  *                 and matrices must stay valid until the last vb_exec_bound using them ends.
- *  vb_exec_bound  enqueues only the GEMM kernel, using the last bound pointers and the
+ *  vb_exec_bound  enqueues only the GEMM kernel(s), using the last bound pointers and the
  *                 given alpha/beta (DEVICE fp32 [batch]).  VB_ERR_INVALID_ARG if never bound.
+ *                 The GEMM kernels reset their own work-list counters when they finish, so
+ *                 vb_exec_bound may be repeated, or captured alone in a CUDA graph and replayed.
  * vb_exec_vbatched(...) == vb_plan_bind(...) + vb_exec_bound(...).
  * ------------------------------------------------------------------------------------ */
 vb_status vb_plan_bind(vb_plan_t plan, const void *const *A, const void *const *B, void *const *C,
