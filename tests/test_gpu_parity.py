@@ -355,3 +355,19 @@ def test_cuda_graph_replays_of_exec_bound(dtype):
             check_batch(db, range(len(M)), SEED, "random")
         else:
             assert all(torch.equal(a, b) for a, b in zip(first, got)), f"replay {rep} differs"
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f16", "f32"])
+@pytest.mark.parametrize("policy", [0, 1])
+def test_random_ragged_shapes(dtype, policy):
+    # 160 GEMMs with M, N, K drawn from [1, 600] (every size class: 1-wide, sub-tile, ragged
+    # multi-tile, K tails), C pre-filled with NaN outside the matrices: every GEMM within the
+    # tolerance and the padding of C never written
+    rng = np.random.default_rng(1234 + policy)
+    r = rng.integers(1, 601, (160, 3))
+    r[:10, 0] = 1
+    r[10:20, 1] = 1
+    r[20:30, 2] = 1
+    db, _ = _run(r[:, 0], r[:, 1], r[:, 2], dtype, policy=policy, seed=5)
+    check_batch(db, range(db.batch), 5, "random")
+    _padding_untouched(db)
