@@ -17,7 +17,10 @@
  *   plan:  tiling engine (§4.2.3, P245-255, Eq. 1) -> tile enumeration ->
  *          batching engine (§5, P259-270: threshold / binary) -> the five auxiliary
  *          arrays of §6 (P282-284, Fig. 6) packed as device tile descriptors.
- *   exec:  one persistent sm_100a kernel walks the descriptors (Fig. 7, P294-312).
+ *   exec:  persistent sm_100a kernels walk the descriptors (Fig. 7, P294-312): tcgen05 for
+ *          bf16/fp16 (a 2-SM cluster launch for pair tiles, then a 1-SM launch), packed-FFMA2
+ *          for fp32.
+ * vb_plan_conv maps a batch of 2-D convolutions onto the same engines (implicit GEMM).
  *
  * Conventions
  *  - Every call returns vb_status; nothing throws across the ABI.  On failure a
@@ -60,7 +63,8 @@ typedef enum {
 /* Strategy tables.
  *  VB_TABLE_V100        PAPER.md Table 2 (P204-214) with the V100 constants (P290):
  *                       TLP threshold 65536, theta 256, versions T = 256 / 128.
- *  VB_TABLE_B200_FFMA   Table 2 shapes for the fp32 FFMA kernel, B200 constants.
+ *  VB_TABLE_B200_FFMA   Table 2 shapes without 128x128 (16x16 ... 128x64 / 64x128) with the
+ *                       128-thread sub-tiles for the fp32 FFMA kernel, T = 128, B200 constants.
  *  VB_TABLE_B200_TC     tcgen05 table (bf16/fp16): 64x32, 128x32, 64x64, 128x64, 64x128,
  *                       128x128, 64x256, 128x256 C tiles and 2-SM pair tiles 256x{64,128,256},
  *                       BK = 64, T = 256; availability tested against max(M, 128) x max(N, 256)
