@@ -799,7 +799,7 @@ extern "C" vb_status vb_plan_info(vb_plan_t p, int64_t *n_tiles, int64_t *n_bloc
     const bool any = p->block_ptr.size() > 1;
     const int nb = (int)p->block_ptr.size() - 1;
     *launches_per_exec = p->batch == 0 ? 0
-                         : p->dt == VB_F32 ? (any ? 1 : 0)
+                         : p->dt == VB_F32 ? 1 + (any ? 1 : 0)   // prep (tensor maps) + FFMA kernel
                                            : 1 + (p->n_pair_blocks > 0) + (nb - p->n_pair_blocks > 0);  // prep + GEMMs
   }
   return VB_OK;
