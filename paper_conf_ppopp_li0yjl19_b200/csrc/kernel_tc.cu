@@ -56,6 +56,9 @@ constexpr int kPageBytes = 8192;
 #ifndef VB_KB_PREFETCH
 #define VB_KB_PREFETCH 0   // experiment: L2 prefetch of each A/B box this many k-blocks ahead
 #endif
+#ifndef VB_A_PAIR_PREFETCH
+#define VB_A_PAIR_PREFETCH 0   // experiment: L2 prefetch of the A box 2 k-blocks ahead at even k-blocks
+#endif
 // L2 evict-first hints on the C_old loads / C stores.  Measured off by default: with the load
 // hint, C5 read 1.3x its compulsory DRAM bytes (a 500^3 batch: C_old fetched ~1.6x) and ran
 // 6% slower; without it DRAM reads are within 1-2% of the compulsory bytes.
@@ -539,6 +542,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
               ptx::tma_load_2d_hint(dst, map, &sh->full[slot], c0, c1, ab_policy);
 #else
               ptx::tma_load_2d(dst, map, &sh->full[slot], c0, c1);
+#endif
+#if VB_A_PAIR_PREFETCH
+            // even k-blocks: L2-prefetch the A box two k-blocks ahead, so that with the 256-byte L2
+            // promotion DRAM sees 512 contiguous bytes of each A row requested together
+            if (i == 0 && (kb & 1) == 0 && kb + 2 < ti.d.kblocks) ptx::tma_prefetch_2d(mapA, (kb + 2) * kBK, row0);
 #endif
 #if VB_KB_PREFETCH > 0
             // start the DRAM fetch of the same box VB_KB_PREFETCH k-blocks ahead into L2
