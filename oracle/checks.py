@@ -87,16 +87,13 @@ def check_plan_invariants(p: Plan, Ms, Ns, Ks, policy: int, theta: int) -> None:
         for blk in p.blocks:
             if len(blk) > 1:
                 ks = [Kt[t] for t in blk]
-                assert sum(ks[:-1]) < theta
-                assert sum(ks) >= theta or blk[-1] in (n_pair - 1, n_tiles - 1)
+                kw = [max(k, 1) for k in ks]          # K-workload, at least 1 (C-11)
+                assert sum(kw[:-1]) < theta
+                assert sum(kw) >= theta or blk[-1] in (n_pair - 1, n_tiles - 1)
     # tiler trace: each round's strategy per GEMM is at least as late in priority order
-    # (tile area never shrinks); the final strategy fits the GEMM unless nothing fits (C-1, C-4)
+    # (tile area never shrinks).  Which strategies were available (P249, or the B200 pre-pass)
+    # is pinned by hand-derived plans in tests/golden, not re-derived here.
     tr = p.tiling.trace
     pos = {r: i for i, r in enumerate(p.table.order())}
     for (r0, _, _), (r1, _, _) in zip(tr, tr[1:]):
         assert all(pos[b] >= pos[a] for a, b in zip(r0, r1))
-    for g, (m, n) in enumerate(zip(Ms, Ns)):
-        s = p.table.rows[p.tiling.rows[g]]
-        mf, nf = max(m, p.table.min_BY), max(n, p.table.min_BX)
-        fits_any = any(q.BY <= mf and q.BX <= nf for q in p.table.rows)
-        assert (s.BY <= mf and s.BX <= nf) or (not fits_any and p.tiling.rows[g] == p.table.order()[0])

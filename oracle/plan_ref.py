@@ -32,8 +32,6 @@ class Table:
     versions: Tuple[int, ...]            # thread counts T, first = preferred (more TLP)
     tlp_threshold: int                   # default TLP threshold (P253, P290)
     theta: int                           # default batching threshold θ (P259, P290)
-    min_BY: int = 0                      # availability floor (reading C-1b); 0 = the paper's rule
-    min_BX: int = 0
 
     def order(self) -> List[int]:
         """Priority order: smaller tile first (P249); ties by table row (reading C-3)."""
@@ -59,16 +57,14 @@ B200_F32 = Table("b200_ffma", V100.rows[:5], versions=(128,), tlp_threshold=4 * 
 # B200 tcgen05 (bf16/fp16) profile: C-tile shapes sized for tcgen05.mma
 # (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16), plus the skinny shapes
 # 128x32 and 64x256, plus 2-SM pair tiles 256x{64,128,256} (ctas = 2, cta_group::2).  One
-# kernel "version" with T = 256 threads.  Availability floor (C-1b): strategies are tested
-# against max(M, 128) and max(N, 256) — an M = 64 MMA costs the cycles of M = 128 and rows
-# past M are never loaded or stored; an edge tile pays only for the columns it has, so the
-# widest tile is available to every GEMM.
+# kernel "version" with T = 256 threads.  Its step 1 is the B200 pre-pass
+# ``b200_step1`` below (readings C-1b, C-7b), not P249's literal rule.
 B200_TC = Table("b200_tcgen05", (
     Strategy("s", 64, 32, 64), Strategy("n", 128, 32, 64), Strategy("m", 64, 64, 64), Strategy("t", 128, 64, 64),
     Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("x", 64, 256, 64),
     Strategy("h", 128, 256, 64), Strategy("T2", 256, 64, 64, 2), Strategy("L2", 256, 128, 64, 2),
     Strategy("H2", 256, 256, 64, 2)),
-    versions=(256,), tlp_threshold=148 * 256, theta=64, min_BY=128, min_BX=256)
+    versions=(256,), tlp_threshold=148 * 256, theta=64)
 
 TABLES = {1: V100, 2: B200_F32, 3: B200_TC}
 
@@ -95,12 +91,65 @@ class TilingResult:
         return [table.strategy_id(r, self.T) for r in self.rows]
 
 
-def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None, pairs_allowed: bool = True) -> TilingResult:
+def step1_p249(Ms, Ns, table: Table) -> List[List[int]]:
+    """Step 1 of §4.2.3 exactly as P249 states it: a GEMM's available strategies are the
+    table's strategies with BY <= M and BX <= N, in a priority queue, smaller tile first
+    (ties by table row, C-3).  If none fits, the smallest strategy alone (C-4)."""
+    order = table.order()
+    queues = []
+    for M, N in zip(Ms, Ns):
+        q = [r for r in order if table.rows[r].BY <= M and table.rows[r].BX <= N]
+        queues.append(q if q else [order[0]])
+    return queues
+
+
+# B200 pre-pass constants (readings C-1b and C-7b; hardware facts, not paper claims).
+TC_MMA_MIN_ROWS = 128     # a 64-row tcgen05.mma issues in the cycles of a 128-row one
+TC_EDGE_FREE_COLS = 256   # an edge tile's MMA N, TMEM columns and B boxes stop at the GEMM's N
+PAIR_MIN_AI = 128         # flop per compulsory byte at which the 2-SM version is offered
+
+
+def b200_availability(M: int, N: int) -> Tuple[int, int]:
+    """Reading C-1b (B200 tcgen05 table only): the extents a strategy is tested against.
+
+    A tile row count below 128 saves no MMA time (an M = 64 MMA costs the cycles of M = 128) and
+    rows past M are neither loaded nor stored, so availability sees at least 128 rows; an edge
+    tile's MMA N, TMEM columns and B boxes end at the GEMM's N, so a tile up to 256 columns wide
+    costs a narrow GEMM nothing and availability sees at least 256 columns."""
+    return max(M, TC_MMA_MIN_ROWS), max(N, TC_EDGE_FREE_COLS)
+
+
+def pairs_allowed(Ms, Ns, Ks, es: int = 2) -> bool:
+    """Reading C-7b: the 2-SM pair version (cta_group::2) is offered only to batches whose
+    arithmetic intensity 2*sum(MNK) / sum(es*(MK + KN) + 2*es*MN) is at least 128 flop/B, i.e.
+    batches near the compute side of the B200 ridge (~265 flop/B); memory-bound batches keep
+    the 1-SM version so that their compute- and memory-heavy tiles overlap in one kernel.
+    (The C term counts a read and a write of C whatever β is: a batch-level platform rule.)"""
+    flops = sum(2 * m * n * k for m, n, k in zip(Ms, Ns, Ks))
+    nbytes = sum(es * (m * k + k * n) + 2 * es * m * n for m, n, k in zip(Ms, Ns, Ks) if m > 0 and n > 0)
+    return nbytes > 0 and flops >= PAIR_MIN_AI * nbytes
+
+
+def b200_step1(Ms, Ns, table: Table, allow_pairs: bool) -> List[List[int]]:
+    """The B200 tcgen05 pre-pass that replaces P249's step 1 for that table only:
+    P249's rule applied to the extents of ``b200_availability`` (C-1b), over the 1-SM
+    strategies only unless ``allow_pairs`` (C-7b).  Pinned by hand-derived plans in
+    ``tests/golden/b200_examples.json``."""
+    order = [r for r in table.order() if allow_pairs or table.rows[r].ctas == 1]
+    queues = []
+    for M, N in zip(Ms, Ns):
+        mf, nf = b200_availability(M, N)
+        q = [r for r in order if table.rows[r].BY <= mf and table.rows[r].BX <= nf]
+        queues.append(q if q else [order[0]])
+    return queues
+
+
+def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None,
+                  queues: List[List[int]] | None = None) -> TilingResult:
     """The three steps and two exceptions of P249–253.
 
-    1. Per GEMM, a priority queue of the strategies with BY <= M and BX <= N (C-1; the
-       B200 tcgen05 table compares against max(M, 128) and max(N, 256), C-1b),
-       smallest first (P249); if none fits, the smallest strategy alone (C-4).
+    1. Per GEMM, a priority queue of available strategies (``queues``; default: P249's
+       literal rule, ``step1_p249``).
     2. Take one strategy per GEMM: pop, or top if only one is left (exception 1, C-2);
        TLP by Eq. 1 with the current version T.
     3. If TLP > threshold (strict, C-6) repeat step 2; otherwise this is the solution.
@@ -111,14 +160,7 @@ def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None, pairs_allo
        every queue there is nothing larger to try and the current solution stands.
     """
     thr = table.tlp_threshold if threshold is None else threshold
-    order = table.order()
-    if not pairs_allowed:                                             # C-7b
-        order = [r for r in order if table.rows[r].ctas == 1]
-    queues = []
-    for M, N in zip(Ms, Ns):
-        mf, nf = max(M, table.min_BY), max(N, table.min_BX)           # C-1b (0 for the paper's tables)
-        q = [r for r in order if table.rows[r].BY <= mf and table.rows[r].BX <= nf]
-        queues.append(q if q else [order[0]])
+    queues = [list(q) for q in (step1_p249(Ms, Ns, table) if queues is None else queues)]
     vi = 0
     T = table.versions[vi]
     trace = []
@@ -169,7 +211,9 @@ def threshold_batching(tiles: Sequence[Tile], T: int, tlp_threshold: int, theta:
 
     Before opening each new block: TLP = (#unassigned tiles + #assigned blocks) * T.
     If TLP > threshold / 2, fill the new block with tiles (enumeration order) until the sum
-    of their K is not less than θ; otherwise every remaining tile gets its own block.
+    of their K-workloads is not less than θ; otherwise every remaining tile gets its own block.
+    A tile's K-workload is its K, counted as at least 1 (reading C-11: a K = 0 tile still
+    runs its epilogue C = βC, so θ also bounds the number of K = 0 tiles in one block).
     """
     n = len(tiles)
     blocks: List[List[int]] = []
@@ -180,7 +224,7 @@ def threshold_batching(tiles: Sequence[Tile], T: int, tlp_threshold: int, theta:
             blk, sk = [], 0
             while i < n and sk < theta:
                 blk.append(i)
-                sk += tiles[i].K
+                sk += max(tiles[i].K, 1)
                 i += 1
             blocks.append(blk)
         else:
@@ -263,29 +307,29 @@ class Plan:
     enc: Encoded
 
 
-PAIR_MIN_AI = 128     # flop per compulsory byte (reading C-7b)
-
-
-def pairs_allowed(Ms, Ns, Ks, es: int = 2) -> bool:
-    """Reading C-7b: the 2-SM pair version (cta_group::2) is offered only to batches whose
-    arithmetic intensity 2*sum(MNK) / sum(es*(MK + KN) + 2*es*MN) is at least 128 flop/B, i.e.
-    batches near the compute side of the B200 ridge (~265 flop/B); memory-bound batches keep
-    the 1-SM version so that their compute- and memory-heavy tiles overlap in one kernel."""
-    flops = sum(2 * m * n * k for m, n, k in zip(Ms, Ns, Ks))
-    nbytes = sum(es * (m * k + k * n) + 2 * es * m * n for m, n, k in zip(Ms, Ns, Ks) if m > 0 and n > 0)
-    return flops >= PAIR_MIN_AI * nbytes and nbytes > 0
-
-
 def plan(Ms, Ns, Ks, table: Table, policy: int = POLICY_THRESHOLD,
          tlp_threshold: int | None = None, theta: int | None = None, es: int = 2, allow_pairs: bool = True) -> Plan:
-    """allow_pairs=False: 1-SM strategies only (the implicit-GEMM convolution plans)."""
+    """The whole host phase: tiling engine, tile enumeration, batching engine, encoding.
+
+    Tables with pair tiles (the B200 tcgen05 table) take step 1 from the B200 pre-pass
+    ``b200_step1``; every other table uses P249 literally.  allow_pairs=False: 1-SM
+    strategies only (the implicit-GEMM convolution plans).
+
+    Reading C-7b (launch split): pair tiles run in their own cluster launch, enqueued before
+    the 1-SM launch on the same stream.  The two launches never run concurrently, so the
+    batching engine sees two batches: it packs the pair tiles and the 1-SM tiles separately
+    (each in enumeration order; P261's TLP counts the thread blocks of one launch) and the
+    pair blocks come first in Tile[].
+    """
     thr = table.tlp_threshold if tlp_threshold is None else tlp_threshold
     th = table.theta if theta is None else theta
     Ms = [int(v) for v in Ms]; Ns = [int(v) for v in Ns]; Ks = [int(v) for v in Ks]
-    tr = tiling_engine(Ms, Ns, table, thr, allow_pairs and pairs_allowed(Ms, Ns, Ks, es))
+    if table is B200_TC:
+        q = b200_step1(Ms, Ns, table, allow_pairs and pairs_allowed(Ms, Ns, Ks, es))
+    else:
+        q = step1_p249(Ms, Ns, table)
+    tr = tiling_engine(Ms, Ns, table, thr, q)
     all_tiles = enumerate_tiles(Ms, Ns, Ks, tr.rows, table)
-    # 2-SM pair tiles run in their own (cluster) kernel: the batching engine packs the pair
-    # tiles and the single tiles separately (each keeps enumeration order); pair blocks first.
     is_pair = [table.rows[tr.rows[t.gemm]].ctas == 2 for t in all_tiles]
     tiles = [t for t, pp in zip(all_tiles, is_pair) if pp] + [t for t, pp in zip(all_tiles, is_pair) if not pp]
     n_pair = sum(is_pair)

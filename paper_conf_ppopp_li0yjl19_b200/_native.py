@@ -95,7 +95,10 @@ def header_symbols() -> list:
 
 
 def _i32(a) -> np.ndarray:
-    return np.ascontiguousarray(np.asarray(a, dtype=np.int64).astype(np.int32))
+    v = np.asarray(a, dtype=np.int64)
+    if v.size and (v.min() < -2**31 or v.max() >= 2**31):
+        raise ValueError("value outside the int32 range of the C-ABI")
+    return np.ascontiguousarray(v.astype(np.int32))
 
 
 def _ptr(a: np.ndarray, ty):

@@ -392,6 +392,7 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
     g.ldb = ldb[i];
     g.ldc = ldc[i];
     g.row = p->tiling.row[i] | ((s.BY / s.ctas) << 8) | (s.BX << 16);   // per-CTA rows
+    if (!p->conv.empty()) g.row |= kGemmConv;   // upload() encodes no B K-tail map for convolutions
     g.kblocks = (int32_t)cdiv64(K[i], s.BK);
   }
   if (p->dt != VB_F32) {
@@ -610,7 +611,9 @@ extern "C" vb_status vb_plan_from_schedule(int device, vb_dtype dt, int32_t batc
       tiles[(size_t)s] = TileRec{g, tile_y[s], tile_x[s], K[g]};
     }
     // 2-SM pair tiles need their own cluster kernel: blocks must not mix pair and 1-SM tiles,
-    // and the pair blocks must come first
+    // and the pair blocks must come first.  Empty blocks are legal anywhere; the pair launch
+    // covers blocks [0, last pair block + 1), so no non-empty 1-SM block may precede a pair block
+    // (the 1-SM kernel must never see a pair tile, whose 256-row geometry it cannot run).
     int n_pair_blocks = 0;
     bool single_seen = false;
     for (int b = 0; b < n_blocks; ++b) {
@@ -622,7 +625,7 @@ extern "C" vb_status vb_plan_from_schedule(int device, vb_dtype dt, int32_t batc
       }
       if (kind == 2) {
         if (single_seen) return fail(VB_ERR_INVALID_ARG, "2-SM pair blocks must precede 1-SM blocks");
-        ++n_pair_blocks;
+        n_pair_blocks = b + 1;
       } else if (kind == 1) {
         single_seen = true;
       }
@@ -882,6 +885,7 @@ extern "C" vb_status vb_fill_uniform_batch(vb_dtype dt, int32_t batch, const int
                                            const int32_t *ld, void *const *ptrs, const int64_t *gemm_id,
                                            uint64_t seed, int32_t operand, int64_t total_elems, void *stream) {
   if (batch < 0) return fail(VB_ERR_INVALID_ARG, "batch < 0");
+  if (dt != VB_F32 && dt != VB_BF16 && dt != VB_F16) return fail(VB_ERR_INVALID_ARG, "unknown dtype %d", (int)dt);
   if (batch == 0) return VB_OK;
   if (!rows || !cols || !ld || !ptrs || !gemm_id) return fail(VB_ERR_INVALID_ARG, "null array");
   cudaError_t e = launch_fill((int)dt, batch, rows, cols, ld, ptrs, gemm_id, seed, operand, total_elems,

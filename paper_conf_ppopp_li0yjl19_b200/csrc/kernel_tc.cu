@@ -915,7 +915,7 @@ __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
   const int BY = (gp.row >> 8) & 0xFF;
   if (w != MAP_C && w != MAP_C_ST && gp.K <= 0) return;
   if (w == MAP_A_TAIL && gp.M % BY == 0) return;        // map not encoded
-  if (w == MAP_B_TAIL && gp.K % 64 == 0) return;
+  if (w == MAP_B_TAIL && (gp.K % 64 == 0 || (gp.row & kGemmConv))) return;   // mirrors upload()
   if (w == MAP_C_ST && gp.N < 8) return;
   const void *ptr = (w == MAP_A || w == MAP_A_TAIL) ? A[g]
                     : (w == MAP_B || w == MAP_B_TAIL) ? B[g]

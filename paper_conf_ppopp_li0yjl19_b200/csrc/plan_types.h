@@ -19,10 +19,12 @@ static_assert(sizeof(TileSlot) == 8, "TileSlot must stay 8 bytes");
 struct alignas(16) GemmParam {
   int32_t M, N, K;
   int32_t lda, ldb, ldc;
-  int32_t row;       // strategy row in the plan's table
+  int32_t row;       // bits 0-7: strategy row in the plan's table; 8-15: per-CTA BY; 16-25: BX;
+                     // bit 30 (kGemmConv): implicit-GEMM convolution (im2col A, no B K-tail map)
   int32_t kblocks;   // ceil(K / BK)
 };
 static_assert(sizeof(GemmParam) == 32, "GemmParam must stay 32 bytes");
+constexpr int32_t kGemmConv = 1 << 30;
 
 // Kernel arguments (by value).
 struct F32Args {

@@ -119,7 +119,9 @@ std::vector<TileRec> enumerate_tiles(const int32_t *M, const int32_t *N, const i
 Schedule batch_threshold(const std::vector<TileRec> &tiles, int T, int64_t tlp_threshold, int theta) {
   // P261 (garbled; reading C-9): before opening a block, TLP = (unassigned + assigned
   // blocks) * T.  If TLP > threshold/2, fill the block in enumeration order until the sum
-  // of K is not less than theta; otherwise every remaining tile is its own block.
+  // of K is not less than theta; otherwise every remaining tile is its own block.  A tile's
+  // K-workload counts at least 1 (C-11): a K = 0 tile still runs its C = beta*C epilogue, so
+  // theta also bounds how many of them one persistent CTA takes.
   Schedule s;
   const int64_t n = (int64_t)tiles.size();
   s.block_ptr.push_back(0);
@@ -131,7 +133,7 @@ Schedule batch_threshold(const std::vector<TileRec> &tiles, int T, int64_t tlp_t
       int64_t sk = 0;
       while (i < n && sk < theta) {
         s.slot_tile.push_back((int32_t)i);
-        sk += tiles[(size_t)i].K;
+        sk += std::max<int64_t>(tiles[(size_t)i].K, 1);
         ++i;
       }
       s.block_ptr.push_back((int32_t)s.slot_tile.size());

@@ -77,6 +77,35 @@ def test_schedule_validation_rejects_double_cover_and_gaps():
         nv.plan_from_schedule(block_ptr=[0, 1], tile_gemm=[0], tile_y=[1], tile_x=[0], **base)
 
 
+def test_schedule_pair_blocks_with_empty_blocks():
+    """an empty block before the pair blocks must not shift the pair/1-SM split.
+    GEMM 0 runs H2 (row 10, 2-SM pair tile), GEMM 1 runs h (row 7, 1-SM)."""
+    base = dict(M=[256, 128], N=[256, 256], K=[64, 64], lda=[64, 64], ldb=[256, 256], ldc=[256, 256],
+                gemm_row=[10, 7], version_T=256, dtype="bf16", device=-1, table_id=vb.VB_TABLE_B200_TC)
+    one = dict(M=[256], N=[256], K=[64], lda=[64], ldb=[256], ldc=[256], gemm_row=[10], version_T=256,
+               dtype="bf16", device=-1, table_id=vb.VB_TABLE_B200_TC)
+    # [empty, pair]: one pair launch only (prep + pair kernel)
+    p = nv.plan_from_schedule(block_ptr=[0, 0, 1], tile_gemm=[0], tile_y=[0], tile_x=[0], **one)
+    assert p.info()["launches_per_exec"] == 2
+    # [empty, pair, single, empty]: prep + pair + 1-SM
+    p = nv.plan_from_schedule(block_ptr=[0, 0, 1, 2, 2], tile_gemm=[0, 1], tile_y=[0, 0], tile_x=[0, 0], **base)
+    assert p.info()["launches_per_exec"] == 3
+    with pytest.raises(vb.VbError):   # a 1-SM block before a pair block
+        nv.plan_from_schedule(block_ptr=[0, 1, 1, 2], tile_gemm=[1, 0], tile_y=[0, 0], tile_x=[0, 0], **base)
+    with pytest.raises(vb.VbError):   # a block mixing the two versions
+        nv.plan_from_schedule(block_ptr=[0, 2], tile_gemm=[0, 1], tile_y=[0, 0], tile_x=[0, 0], **base)
+
+
+def test_fill_rejects_unknown_dtype():
+    st = nv.lib.vb_fill_uniform_batch(7, 0, None, None, None, None, None, 0, 0, 0, None)
+    assert st == vb.VB_ERR_INVALID_ARG
+
+
+def test_int32_range_checked_before_the_abi():
+    with pytest.raises(ValueError):
+        nv.plan_vbatched([8], [8], [2**32 + 16], [8], [8], [8], "bf16", device=-1)
+
+
 def test_validation_errors():
     with pytest.raises(vb.VbError) as e:
         nv.plan_vbatched([8], [8], [8], [9], [8], [8], "bf16", device=-1)   # lda*2 not a 16-B multiple

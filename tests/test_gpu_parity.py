@@ -286,13 +286,6 @@ def test_pair_tiles_selected_for_compute_bound_batch(dtype):
     _padding_untouched(db)
 
 
-def test_memory_bound_batch_keeps_one_sm_tiles():
-    M, N, K = vbinputs.config_sizes("C5")
-    assert not pr.pairs_allowed(M, N, K)
-    M, N, K = vbinputs.config_sizes("C4")
-    assert pr.pairs_allowed(M, N, K)
-
-
 # ------------------------------------------------------------------ policy selection (P272-274)
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])
 def test_auto_policy_parity(dtype):
