@@ -181,6 +181,20 @@ def roofline_for(dtype, flops, nbytes, t_s, peaks, sustained=False):
             "frac": (flops / t_s) / p, "t_roof_us": t_c * 1e6}
 
 
+def aggregate_roofline(dtype, flops_all, bytes_all, makespan_s, t_roof_max_us, world, peaks):
+    """N > 1: the job's roofline is the slowest rank's t_roof; `frac` is the
+    whole-job achieved rate over N times the per-GPU peak (= sum of the ranks' bytes or flops /
+    makespan / (N * peak)), and `frac_makespan` = max over ranks of t_roof / makespan."""
+    r = roofline_for(dtype, flops_all, bytes_all, makespan_s, peaks)
+    one = r["peak"]
+    r["peak"] = one * world
+    r["frac"] = r["achieved"] / r["peak"]
+    r["t_roof_us"] = t_roof_max_us
+    r["frac_makespan"] = t_roof_max_us * 1e-6 / makespan_s
+    r["aggregate"] = f"{world} ranks: achieved = sum over ranks / makespan, peak = {world} x {one}"
+    return r
+
+
 def committed_traffic(cfg):
     """dram read+write bytes per launch from the committed ncu capture (profiles/), or None."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -310,14 +324,17 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
     clk = clocks.stop() if clocks else None
     step_ms = sum(s.elapsed_time(e) for s, e in zip(starts, ends)) / steps
     kern_ms = sum(m.elapsed_time(e) for m, e in zip(mids, ends)) / steps
-    step_ms_max, kern_ms_max, plan_ms_max = gather_max([step_ms, kern_ms, plan_ms], world, dist_device)
+    t_roof_rank = roofline_for(dtype, flops, nbytes, 1.0, peaks)["t_roof_us"]
+    step_ms_max, kern_ms_max, plan_ms_max, t_roof_max = gather_max([step_ms, kern_ms, plan_ms, t_roof_rank], world,
+                                                                    dist_device)
     flops_all, bytes_all = gather_sum([float(flops), float(nbytes)], world, dist_device)
     res = {
         "cfg": cfg, "dtype": dtype, "flops_rank": flops, "bytes_rank": nbytes, "flops": flops_all,
         "step_ms": step_ms_max, "kernel_ms": kern_ms_max, "plan_ms": plan_ms_max,
         "value": flops_all / (step_ms_max * 1e-3) / 1e12,
         "kernel_tflops": flops_all / (kern_ms_max * 1e-3) / 1e12,
-        "roofline": roofline_for(dtype, flops, nbytes, kern_ms * 1e-3, peaks),
+        "roofline": roofline_for(dtype, flops, nbytes, kern_ms * 1e-3, peaks) if world == 1 else
+        aggregate_roofline(dtype, flops_all, bytes_all, kern_ms_max * 1e-3, t_roof_max, world, peaks),
         "plan": pinfo, "policy_chosen": {0: "threshold", 1: "binary", 2: "none"}.get(plan.policy(), "?"), "l2": "flushed (512 MB write) between steps" if small else
         f"inputs ({db.arena_bytes() / 1e9:.1f} GB per rank) >> L2 (126 MB); no flush",
         "launches": pinfo["launches_per_exec"] * steps, "clocks": clk, "batch_rank": int(db.batch),
@@ -490,13 +507,16 @@ def main_ours(args):
                 aux[cfg]["cuda_graph_step_ms"] = round(r["graph_step_ms"], 4)
             del d2, p2
             torch.cuda.empty_cache()
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()          # every rank's GPU work is done: rank 0 times the oracle on idle cores
+    if rank == 0 and not args.no_cpu_baseline:
         info = vbinputs.CONFIGS[args.config]
         M, N, K = vbinputs.config_sizes(args.config, nb=args.nb if args.config == "C3" else 1)
         cpu = time_oracle(M, N, K, info["dtype"], info["ab"], args.seed, seconds=args.cpu_seconds)
         cpu.pop("ms_per_step", None)
     rl = res["roofline"]
-    rl["traffic"] = committed_traffic(args.config)
+    rl["traffic"] = committed_traffic(args.config) if world == 1 else None   # ncu capture is of the 1-GPU launch
     rl_out = _round(rl)
     rl_out["kernel"] = "vb_tc_kernel (persistent tcgen05 GEMM)" if res["dtype"] != "f32" else "vb_f32_kernel (FFMA)"
     rl_out["peak_source"] = f"{peaks['_source']} (MEASURED_PEAKS.json)" if peaks["_source"] == "measured" else \
@@ -561,6 +581,19 @@ def main_reference(args):
     return 0
 
 
+def spawn_ranks(n, argv):
+    """`bench.py --gpus N` without a launcher: start N ranks (one process per GPU) through
+    torch.distributed.run on 127.0.0.1, exactly as the driver's torchrun launch would, and
+    return their exit status (rank 0 prints the JSON line)."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + argv
+    return subprocess.call(cmd)
+
+
 def main(argv=None):
     ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
     ap.add_argument("--gpus", type=int, default=1)
@@ -578,6 +611,8 @@ def main(argv=None):
     ap.add_argument("--no-aux", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args(argv)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return spawn_ranks(args.gpus, sys.argv[1:] if argv is None else list(argv))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     if world != args.gpus and args.impl == "ours":
         print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}; using WORLD_SIZE", file=sys.stderr)

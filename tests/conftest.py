@@ -18,3 +18,14 @@ def golden():
     import json
     with open(os.path.join(ROOT, "tests", "golden", "paper_examples.json")) as f:
         return json.load(f)
+
+
+def pytest_sessionfinish(session, exitstatus):
+    mod = sys.modules.get("gpu_helpers")
+    rec = getattr(mod, "RECORD", None) if mod else None
+    if rec:
+        import json
+        out = os.environ.get("VB_PARITY_OUT", os.path.join(ROOT, "gpurun_out", "parity.json"))
+        os.makedirs(os.path.dirname(out), exist_ok=True)
+        with open(out, "w") as f:
+            json.dump({"exitstatus": int(exitstatus), "cases": rec}, f, indent=1, sort_keys=True)

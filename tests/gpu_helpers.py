@@ -7,7 +7,11 @@ import torch
 
 import vbinputs
 from oracle import gemm as og
-from oracle.checks import TOL, normwise_error
+from oracle.checks import TOL, normwise_error, significant_rel_error
+
+# achieved errors per named case, written by tests/conftest.py at session end to
+# $VB_PARITY_OUT (default gpurun_out/parity.json) when any test recorded one
+RECORD: dict = {}
 
 
 def to_f64(t: torch.Tensor) -> np.ndarray:
@@ -67,3 +71,35 @@ def check_bound(db, idx, seed, ab_mode, c_old=None):
         bad = err > bound
         assert not bad.any(), (f"GEMM {g} (M,N,K)=({m},{n},{k}): {int(bad.sum())} elements outside the error "
                                f"bound, worst excess {float((err - bound).max()):.3e}")
+
+
+def check_recorded(name, db, idx, seed, ab_mode, c_old=None):
+    """Normwise tolerance AND the elementwise bound on GEMMs idx, and record the achieved
+    errors under `name`: worst normwise error, worst err/bound ratio, worst significant
+    elementwise relative error (C-18), and how many GEMMs / elements were checked."""
+    refs = oracle_for(db, idx, seed, ab_mode, c_old)
+    al, be = vbinputs.alpha_beta(seed, db.gemm_ids[list(idx)], ab_mode)
+    tol = TOL[db.dtype]
+    worst_nw = worst_ratio = worst_sig = 0.0
+    n_el = 0
+    for t, (g, ref) in enumerate(zip(idx, refs)):
+        m, n, k = int(db.M[g]), int(db.N[g]), int(db.K[g])
+        got = to_f64(db.c(g))
+        nw = normwise_error(got, ref)
+        assert nw <= tol, f"{name}: GEMM {g} (M,N,K)=({m},{n},{k}): normwise error {nw:.3e} > {tol}"
+        a, b, c = host_inputs(seed, int(db.gemm_ids[g]), m, n, k, db.dtype)
+        if c_old is not None:
+            c = np.asarray(c_old[t], np.float64)
+        mag = [np.abs(c).copy()]
+        og.gemm_batch([np.abs(a)], [np.abs(b)], mag, [abs(float(al[t]))], [abs(float(be[t]))])
+        bound = (k + 2) * 2.0 ** -24 * mag[0] + U_OUT[db.dtype] * np.abs(ref) + 2.0 ** -24
+        err = np.abs(got - ref)
+        ratio = float((err / bound).max()) if err.size else 0.0
+        assert ratio <= 1.0, f"{name}: GEMM {g} (M,N,K)=({m},{n},{k}): {int((err > bound).sum())} elements outside the bound"
+        worst_nw, worst_ratio = max(worst_nw, nw), max(worst_ratio, ratio)
+        worst_sig = max(worst_sig, significant_rel_error(got, ref))
+        n_el += err.size
+    RECORD[name] = {"dtype": db.dtype, "gemms_checked": len(list(idx)), "elements_checked": int(n_el),
+                    "normwise_max": worst_nw, "tolerance": tol, "bound_ratio_max": worst_ratio,
+                    "significant_rel_max": worst_sig}
+    return RECORD[name]

@@ -7,7 +7,7 @@ import torch
 
 import vbinputs
 from oracle import plan_ref as pr
-from gpu_helpers import check_batch, check_bound, to_f64
+from gpu_helpers import check_batch, check_bound, check_recorded, to_f64
 
 pytestmark = pytest.mark.gpu
 
@@ -72,7 +72,7 @@ def test_c1_fp32_v100_profile_and_128_threads():
 def test_c2_fp32_full():
     M, N, K = vbinputs.config_sizes("C2")
     db, _ = _run(M, N, K, "f32", 0)
-    check_batch(db, range(db.batch), SEED, "random")
+    check_recorded("C2/threshold-full", db, range(db.batch), SEED, "random")
     _padding_untouched(db)
 
 
@@ -104,7 +104,7 @@ EDGE = [(1, 1, 1), (5, 3, 7), (64, 32, 64), (65, 33, 65), (127, 63, 1), (129, 65
 def test_tc_edge_shapes(dtype, policy):
     M, N, K = (np.array(c) for c in zip(*EDGE))
     db, _ = _run(M, N, K, dtype, policy)
-    check_batch(db, range(db.batch), SEED, "random")
+    check_recorded(f"edge/{dtype}/p{policy}", db, range(db.batch), SEED, "random")
     _padding_untouched(db)
 
 
@@ -179,7 +179,7 @@ def _sampled(cfg, n_sample, policy=0):
     rng = np.random.default_rng(7)
     idx = sorted(set([int(np.argmax(work)), int(np.argmin(work)), 0, len(M) - 1] +
                      list(rng.choice(len(M), n_sample, replace=False))))
-    return check_batch(db, idx, SEED, "random")
+    return check_recorded(f"{cfg}-sampled/p{policy}", db, idx, SEED, "random")
 
 
 def test_c4_sampled_full_size():
@@ -362,5 +362,5 @@ def test_random_ragged_shapes(dtype, policy):
     r[10:20, 1] = 1
     r[20:30, 2] = 1
     db, _ = _run(r[:, 0], r[:, 1], r[:, 2], dtype, policy=policy, seed=5)
-    check_batch(db, range(db.batch), 5, "random")
+    check_recorded(f"ragged160/{dtype}/p{policy}", db, range(db.batch), 5, "random")
     _padding_untouched(db)
