@@ -276,9 +276,16 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
         db = DeviceBatch(M[idx], N[idx], K[idx], dtype, device=dev, gemm_ids=idx)
     db.fill(args.seed, ab)
     torch.cuda.synchronize(dev)
-    t0 = time.perf_counter()
-    plan = db.plan(vb.POLICIES[args.policy])
-    plan_ms = (time.perf_counter() - t0) * 1e3
+    # planning cost (host tiling + batching engines, device descriptor expansion, tensor maps):
+    # the first plan of the process, then the steady state of re-planning (the paper's on-line
+    # case, P272-274), median of 5; the last plan is the one that runs
+    plan_times = []
+    for _ in range(6):
+        t0 = time.perf_counter()
+        plan = db.plan(vb.POLICIES[args.policy])
+        plan_times.append((time.perf_counter() - t0) * 1e3)
+    plan_ms = float(np.median(plan_times[1:]))
+    plan_first_ms = plan_times[0]
     pinfo = plan.info()
     flops = db.flops()
     beta_nz = db.beta[:db.batch].cpu().numpy() != 0
@@ -330,7 +337,7 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
     flops_all, bytes_all = gather_sum([float(flops), float(nbytes)], world, dist_device)
     res = {
         "cfg": cfg, "dtype": dtype, "flops_rank": flops, "bytes_rank": nbytes, "flops": flops_all,
-        "step_ms": step_ms_max, "kernel_ms": kern_ms_max, "plan_ms": plan_ms_max,
+        "step_ms": step_ms_max, "kernel_ms": kern_ms_max, "plan_ms": plan_ms_max, "plan_first_ms": plan_first_ms,
         "value": flops_all / (step_ms_max * 1e-3) / 1e12,
         "kernel_tflops": flops_all / (kern_ms_max * 1e-3) / 1e12,
         "roofline": roofline_for(dtype, flops, nbytes, kern_ms * 1e-3, peaks) if world == 1 else
@@ -532,7 +539,8 @@ def main_ours(args):
             "parallelism": f"gemm-sharded x{world} (LPT on 2MNK, no data-path collective)" if world > 1 else
             "single GPU", "policy": args.policy if args.policy != "auto" else
             f"auto (random forest, P272-274) -> {res['policy_chosen']}", "table": "b200_tcgen05" if res["dtype"] != "f32" else "b200_ffma",
-            "l2": res["l2"], "plan_ms": round(res["plan_ms"], 2), "n_tiles_rank0": res["plan"]["n_tiles"],
+            "l2": res["l2"], "plan_ms": round(res["plan_ms"], 2), "plan_first_ms": round(res["plan_first_ms"], 2),
+            "n_tiles_rank0": res["plan"]["n_tiles"],
             "n_blocks_rank0": res["plan"]["n_blocks"], "kernel_ms": round(res["kernel_ms"], 4),
             "kernel_tflops": round(res["kernel_tflops"], 3)},
         "roofline": rl_out,

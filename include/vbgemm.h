@@ -231,6 +231,14 @@ vb_status vb_plan_tune(int device, vb_dtype dt, int32_t batch,
 vb_status vb_plan_export(vb_plan_t plan, int32_t *block_ptr, int32_t *tile_gemm,
                          int32_t *tile_y, int32_t *tile_x, int32_t *gemm_strategy);
 
+/* vb_plan_debug_tmaps — diagnostic: copy the plan's per-GEMM tensor maps (DEVICE copy,
+ * batch x 6 x 128 bytes for bf16/fp16 plans, batch x 2 x 128 for fp32) to the HOST buffer `out`
+ * of `bytes` bytes; *needed receives the size (0 for host-only plans).  Tests use it to check
+ * that maps built on the device from templates equal the host encoder's maps bit for bit
+ * (the environment variable VB_TMAPS_HOST=1 makes vb_plan_* encode every map on the host).
+ * Errors: VB_ERR_INVALID_ARG (null plan, buffer too small), VB_ERR_CUDA. */
+vb_status vb_plan_debug_tmaps(vb_plan_t plan, void *out, int64_t bytes, int64_t *needed);
+
 /* vb_plan_tiler_trace — per round of the tiling engine: TLP (Eq. 1) and version T.
  * Writes min(cap, rounds) entries; *n_rounds receives the total number of rounds. */
 vb_status vb_plan_tiler_trace(vb_plan_t plan, int32_t cap, int64_t *tlp, int32_t *version_T,

@@ -64,6 +64,7 @@ lib.vb_plan_info.argtypes = [_vp, _i64p, _i64p, _i64p, _i32p, _i32p]
 lib.vb_plan_export.argtypes = [_vp, _i32p, _i32p, _i32p, _i32p, _i32p]
 lib.vb_plan_tiler_trace.argtypes = [_vp, ctypes.c_int32, _i64p, _i32p, _i32p]
 lib.vb_plan_destroy.argtypes = [_vp]
+lib.vb_plan_debug_tmaps.argtypes = [_vp, _vp, ctypes.c_int64, _i64p]
 lib.vb_plan_policy.argtypes = [_vp, _i32p]
 lib.vb_plan_tune.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int32] + [_i32p] * 6 + \
     [_P(vb_tuning), _vp, _vp, _vp, _vp, _vp, ctypes.c_int32, _vp, _P(_vp), _P(ctypes.c_float)]
@@ -74,7 +75,7 @@ lib.vb_fill_alpha_beta.argtypes = [ctypes.c_int32, _vp, ctypes.c_uint64, _vp, _v
 lib.vb_device_info.argtypes = [ctypes.c_int, _i32p, _i32p, _i32p]
 for _f in ("vb_plan_vbatched", "vb_plan_from_schedule", "vb_exec_vbatched", "vb_plan_bind", "vb_exec_bound", "vb_plan_info", "vb_plan_export",
            "vb_plan_tiler_trace", "vb_plan_destroy", "vb_plan_policy", "vb_plan_tune", "vb_shard_lpt", "vb_fill_uniform_batch", "vb_fill_alpha_beta",
-           "vb_device_info"):
+           "vb_device_info", "vb_plan_debug_tmaps"):
     getattr(lib, _f).restype = ctypes.c_int
 
 
@@ -149,6 +150,15 @@ class Plan:
                                  _ptr(gs, _i32p)))
         return dict(block_ptr=bp, tile_gemm=tg[:n], tile_y=ty[:n], tile_x=tx[:n], gemm_strategy=gs[:self.batch],
                     version_T=inf["version_T"])
+
+    def debug_tmaps(self) -> np.ndarray:
+        """The plan's tensor maps (device copy) as raw bytes [batch, maps, 128] (diagnostic)."""
+        n = ctypes.c_int64()
+        check(lib.vb_plan_debug_tmaps(self.handle, None, 0, ctypes.byref(n)))
+        out = np.zeros(n.value, np.uint8)
+        if n.value:
+            check(lib.vb_plan_debug_tmaps(self.handle, out.ctypes.data, n.value, ctypes.byref(n)))
+        return out.reshape(self.batch, -1, 128) if n.value else out
 
     def tiler_trace(self):
         n = ctypes.c_int32()

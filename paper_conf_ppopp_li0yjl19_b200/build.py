@@ -15,7 +15,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libvbgemm.so")
 TRACE_LIB = os.path.join(HERE, "libvbgemm_trace.so")
-SOURCES = ["capi.cu", "planner.cpp", "forest.cpp", "kernel_f32.cu", "kernel_tc.cu", "fill.cu"]
+SOURCES = ["capi.cu", "planner.cpp", "forest.cpp", "kernel_f32.cu", "kernel_tc.cu", "fill.cu", "plan_dev.cu"]
 HEADERS = ["tables.h", "planner.h", "plan_types.h", "sm100.cuh", "forest.h", "forest_b200.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",

@@ -94,6 +94,52 @@ struct TcArgs {
   const ConvParam *conv;    // [batch] for convolution plans (vb_plan_conv), else nullptr
 };
 
+// Plan-time expansion of the compact schedule (csrc/plan_dev.cu).
+struct ExpandArgs {
+  const int32_t *slot_tile;   // [n_slots] slot -> tile in enumeration order; nullptr = identity
+  const int32_t *seg_start;   // [n_seg + 1] first tile of each GEMM segment (enumeration order)
+  const int32_t *seg_gemm;    // [n_seg] GEMM of each segment (GEMMs without tiles have none)
+  int32_t n_seg;
+  int64_t n_slots;
+  const GemmParam *gemms;
+  const ConvParam *conv;      // [batch] for convolution plans, else nullptr
+  TileDesc *tiles;            // tensor-core plans: TileDesc[n_slots] (else nullptr)
+  TileSlot *slots;            // FFMA plans: TileSlot[n_slots] (else nullptr)
+  int16_t row_by[16], row_bx[16];   // full tile extents (BY, BX) of each table row
+};
+
+// Plan-time construction of the per-GEMM tensor maps from host-encoded templates.
+// A map's template is tidx[map][row][box_outer / 8][small] (kTmapKeys entries, -1 = none):
+// the box follows from the strategy row, the tail rows of A (M % BY) and B (K % 64), and `small`
+// is the encoder's size class (tensor spans < kTmapSmallBytes from first to last element).
+constexpr int kTmapKeys = 6 * 16 * 33 * 2;
+constexpr uint64_t kTmapSmallBytes = 128 * 1024;
+__host__ __device__ inline int tmap_key(int w, int row, int box_outer, bool small) {
+  return ((w * 16 + row) * 33 + box_outer / 8) * 2 + (small ? 1 : 0);
+}
+struct MapBuildArgs {
+  uint8_t *tmaps;             // CUtensorMap[batch][kMapsPerGemm]
+  const uint8_t *templates;   // CUtensorMap[n_templates]
+  const int16_t *tidx;        // [kTmapKeys] template index by tmap_key
+  const GemmParam *gemms;
+  int32_t batch;
+  int32_t es;                 // element bytes
+};
+
+// Box rows (outer extent) of map w of a tensor-core GEMM, or 0 when the map is not used
+// (the conditions of the kernels' map selection and of the bind-time prep kernel).
+__host__ __device__ inline int tc_map_outer(int w, int M, int N, int K, int BYc) {
+  if (M <= 0 || N <= 0) return 0;
+  switch (w) {
+    case 0: return K > 0 ? BYc : 0;                                              // A
+    case 1: return (K > 0 && M % BYc) ? (M % BYc + 7) / 8 * 8 : 0;               // A row tail
+    case 2: return K > 0 ? 64 : 0;                                               // B
+    case 3: return (K > 0 && K % 64) ? (K % 64 + 15) / 16 * 16 : 0;              // B K tail
+    case 4: return BYc / 4;                                                      // C (loads)
+    default: return N >= 8 ? BYc / 4 : 0;                                        // C store
+  }
+}
+
 // Tensor-core strategy geometry derived from a table row (BY, BX): TMA boxes and swizzles.
 struct TcGeom {
   int BY, BX;

@@ -25,9 +25,20 @@ struct TileRec {
   int32_t gemm, y, x, K;
 };
 
-struct Schedule {                  // the five auxiliary arrays of Fig. 6 (P282)
+struct Schedule {                  // the batching scheme (Fig. 6, P282)
   std::vector<int32_t> block_ptr;  // Tile[]  (Block_NUM + 1)
-  std::vector<int32_t> slot_tile;  // slot -> tile index (enumeration order)
+  std::vector<int32_t> slot_tile;  // slot -> tile (enumeration order); EMPTY = identity (threshold, none)
+};
+
+// The tile enumeration in compact form: GEMM gemm[j] owns tiles [start[j], start[j+1]) in
+// row-major (y, x) order.  Segments [0, n_pair) are the GEMMs on 2-SM pair strategies.
+struct Segments {
+  std::vector<int32_t> gemm;
+  std::vector<int64_t> start;      // [n_seg + 1]
+  int n_pair = 0;
+  int64_t n_pair_tiles = 0;
+  int64_t n_tiles() const { return start.empty() ? 0 : start.back(); }
+  int64_t find(int64_t tile) const;
 };
 
 // Eq. 1 (P220) with ceil tile counts (reading C-5); a 2-SM pair tile counts twice.
@@ -42,15 +53,22 @@ TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const Tab
 // 2*sum(MNK) / sum(es*(MK+KN) + 2*es*MN) >= 128 flop/byte.
 bool pairs_allowed(const int32_t *M, const int32_t *N, const int32_t *K, int batch, int elem_bytes);
 
-// GEMM-major, row-major (y, x) tiles (P133-135, P157, P284; C-11, C-13).
-std::vector<TileRec> enumerate_tiles(const int32_t *M, const int32_t *N, const int32_t *K,
-                                     int batch, const std::vector<int> &row, const TableDef &t);
+// GEMM-major, row-major (y, x) tiles (P133-135, P157, P284; C-11, C-13), pair-strategy GEMMs
+// first (reading C-7b), as segments.
+Segments build_segments(const int32_t *M, const int32_t *N, int batch, const std::vector<int> &row,
+                        const TableDef &t);
+// (GEMM, Y, X, K) of one tile of the enumeration (host mirror of the device expansion).
+TileRec decode_tile(const Segments &sg, const int32_t *N, const int32_t *K, const std::vector<int> &row,
+                    const TableDef &t, int64_t tile);
 
-// Threshold batching (P261, reading C-9), binary batching (P263-270, Eq. 5, reading C-10),
-// and one tile per block.
-Schedule batch_threshold(const std::vector<TileRec> &tiles, int T, int64_t tlp_threshold, int theta);
-Schedule batch_binary(const std::vector<TileRec> &tiles, int theta);
-Schedule batch_none(const std::vector<TileRec> &tiles);
+// Batching of one launch's tiles (part 0: pair tiles, 1: 1-SM tiles), appended to s
+// (s.block_ptr must already hold its leading entry): threshold batching (P261, reading C-9),
+// binary batching (P263-270, Eq. 5, reading C-10) and one tile per block.  Threshold and none
+// keep the enumeration order (s.slot_tile stays empty); binary fills s.slot_tile.
+void batch_threshold(const Segments &sg, const int32_t *K, int part, int T, int64_t tlp_threshold, int theta,
+                     Schedule &s);
+void batch_binary(const Segments &sg, const int32_t *K, int part, int theta, Schedule &s);
+void batch_none(const Segments &sg, int part, Schedule &s);
 
 // LPT on 2*M*N*K (BASELINE.json; reading C-23).
 std::vector<int32_t> shard_lpt(const int32_t *M, const int32_t *N, const int32_t *K, int batch,

@@ -364,3 +364,38 @@ def test_random_ragged_shapes(dtype, policy):
     db, _ = _run(r[:, 0], r[:, 1], r[:, 2], dtype, policy=policy, seed=5)
     check_recorded(f"ragged160/{dtype}/p{policy}", db, range(db.batch), 5, "random")
     _padding_untouched(db)
+
+
+@pytest.mark.parametrize("cfg", ["C4", "ragged"])
+def test_device_built_tensor_maps_equal_host_encoded(cfg, monkeypatch):
+    """Plan-time tensor maps built on the device (templates + tensormap.replace of the global
+    dims and stride) are bit-identical to cuTensorMapEncodeTiled's maps for every GEMM and map,
+    once both plans are bound to the same buffers (the bind patches the address)."""
+    if cfg == "C4":
+        M, N, K = vbinputs.config_sizes("C4")
+    else:
+        r = np.random.default_rng(21).integers(1, 700, (300, 3))
+        r[:20, 2] = 0
+        r[20:40, 1] = np.random.default_rng(2).integers(1, 8, 20)
+        # tensors spanning just below / exactly / above 128 KiB (rows x row stride), with and
+        # without row padding: the encoder's size class (DESIGN.md §5)
+        edge = np.array([[1024, 40, 64], [1023, 40, 64], [1024, 40, 63], [1025, 40, 63], [40, 64, 1024],
+                         [40, 64, 1023], [40, 63, 1024], [1024, 64, 40], [1023, 64, 40], [1024, 57, 40]])
+        r = np.concatenate([r, edge])
+        M, N, K = r[:, 0], r[:, 1], r[:, 2]
+    db = DeviceBatch(M, N, K, "bf16")
+    db.fill(SEED)
+    dev_plan = db.plan()
+    monkeypatch.setenv("VB_TMAPS_HOST", "1")
+    host_plan = db.plan()
+    monkeypatch.delenv("VB_TMAPS_HOST")
+    for p in (dev_plan, host_plan):
+        db.bind(p)
+    torch.cuda.synchronize()
+    a, b = dev_plan.debug_tmaps(), host_plan.debug_tmaps()
+    assert a.shape == b.shape and a.shape[0] == len(M)
+    bad = np.nonzero((a != b).any(axis=2))
+    assert bad[0].size == 0, f"{bad[0].size} maps differ, first GEMM {bad[0][:5]} map {bad[1][:5]}"
+    db.run(dev_plan)
+    torch.cuda.synchronize()
+    check_batch(db, range(0, len(M), max(1, len(M) // 60)), SEED, "random")
