@@ -228,12 +228,14 @@ def oracle_sample(M, N, K, dtype, ab_mode, seed, rng, target_flops):
 def time_oracle(M, N, K, dtype, ab_mode, seed, seconds=10.0, steps=1, warmup=0):
     """Time the fp64 oracle (as it stands) on a bounded sample; returns a result dict."""
     from oracle import gemm as og
-    cores = og.max_threads()
+    # every host core: torchrun sets OMP_NUM_THREADS=1 per rank, but the oracle runs on rank 0
+    # alone after the GPU work of every rank is done
+    cores = os.cpu_count() or og.max_threads()
     rng = np.random.default_rng(12345)
     # calibrate the rate on a small sample, then size the per-step sample for `seconds`
     pick, As, Bs, Cs, al, be, f0 = oracle_sample(M, N, K, dtype, ab_mode, seed, rng, 2e9)
     t0 = time.perf_counter()
-    og.gemm_batch(As, Bs, [c.copy() for c in Cs], al, be)
+    og.gemm_batch(As, Bs, [c.copy() for c in Cs], al, be, nthreads=cores)
     rate = f0 / max(time.perf_counter() - t0, 1e-6)
     pick, As, Bs, Cs, al, be, fl = oracle_sample(M, N, K, dtype, ab_mode, seed, np.random.default_rng(777),
                                                  rate * seconds)
@@ -241,7 +243,7 @@ def time_oracle(M, N, K, dtype, ab_mode, seed, seconds=10.0, steps=1, warmup=0):
     for it in range(warmup + steps):
         cw = [c.copy() for c in Cs]
         t0 = time.perf_counter()
-        og.gemm_batch(As, Bs, cw, al, be)
+        og.gemm_batch(As, Bs, cw, al, be, nthreads=cores)
         dt = time.perf_counter() - t0
         if it >= warmup:
             times.append(dt)

@@ -239,6 +239,15 @@ vb_status vb_plan_export(vb_plan_t plan, int32_t *block_ptr, int32_t *tile_gemm,
  * Errors: VB_ERR_INVALID_ARG (null plan, buffer too small), VB_ERR_CUDA. */
 vb_status vb_plan_debug_tmaps(vb_plan_t plan, void *out, int64_t bytes, int64_t *needed);
 
+/* vb_debug_set_coverage — diagnostic, coverage-counter build only (libvbgemm_cov.so, compiled
+ * with -DVB_COVERAGE; SURVEY.md §4 "each C element written exactly once"): from now on every
+ * element a GEMM kernel's epilogue stores on `device` also adds 1 to the int32 counter at the
+ * same element offset from `c_base` in the DEVICE array `counts` (caller-owned, zeroed by the
+ * caller, one counter per element of the C arena that starts at `c_base`, element size
+ * `elem_bytes`).  counts = NULL switches counting off.  The product build returns
+ * VB_ERR_UNSUPPORTED; VB_ERR_INVALID_ARG for a missing base or element size. */
+vb_status vb_debug_set_coverage(int device, int32_t *counts, const void *c_base, int32_t elem_bytes);
+
 /* vb_plan_tiler_trace — per round of the tiling engine: TLP (Eq. 1) and version T.
  * Writes min(cap, rounds) entries; *n_rounds receives the total number of rounds. */
 vb_status vb_plan_tiler_trace(vb_plan_t plan, int32_t cap, int64_t *tlp, int32_t *version_T,

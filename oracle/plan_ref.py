@@ -52,7 +52,7 @@ V100 = Table("v100_table2", (
 # B200 FFMA (fp32) profile: the Table 2 shapes (an FFMA design) without the 128x128 row, one
 # version with T = 128 threads; platform constants re-set for 148 SMs (calibrated on B200,
 # DESIGN.md §4 and §6.2, reading C-22).
-B200_F32 = Table("b200_ffma", V100.rows[:5], versions=(128,), tlp_threshold=4 * 148 * 256, theta=64)
+B200_F32 = Table("b200_ffma", V100.rows[:5], versions=(128,), tlp_threshold=2 * 148 * 256, theta=64)
 
 # B200 tcgen05 (bf16/fp16) profile: C-tile shapes sized for tcgen05.mma
 # (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16), plus the skinny shapes

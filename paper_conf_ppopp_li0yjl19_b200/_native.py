@@ -65,6 +65,7 @@ lib.vb_plan_export.argtypes = [_vp, _i32p, _i32p, _i32p, _i32p, _i32p]
 lib.vb_plan_tiler_trace.argtypes = [_vp, ctypes.c_int32, _i64p, _i32p, _i32p]
 lib.vb_plan_destroy.argtypes = [_vp]
 lib.vb_plan_debug_tmaps.argtypes = [_vp, _vp, ctypes.c_int64, _i64p]
+lib.vb_debug_set_coverage.argtypes = [ctypes.c_int, _vp, _vp, ctypes.c_int32]
 lib.vb_plan_policy.argtypes = [_vp, _i32p]
 lib.vb_plan_tune.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int32] + [_i32p] * 6 + \
     [_P(vb_tuning), _vp, _vp, _vp, _vp, _vp, ctypes.c_int32, _vp, _P(_vp), _P(ctypes.c_float)]
@@ -75,7 +76,7 @@ lib.vb_fill_alpha_beta.argtypes = [ctypes.c_int32, _vp, ctypes.c_uint64, _vp, _v
 lib.vb_device_info.argtypes = [ctypes.c_int, _i32p, _i32p, _i32p]
 for _f in ("vb_plan_vbatched", "vb_plan_from_schedule", "vb_exec_vbatched", "vb_plan_bind", "vb_exec_bound", "vb_plan_info", "vb_plan_export",
            "vb_plan_tiler_trace", "vb_plan_destroy", "vb_plan_policy", "vb_plan_tune", "vb_shard_lpt", "vb_fill_uniform_batch", "vb_fill_alpha_beta",
-           "vb_device_info", "vb_plan_debug_tmaps"):
+           "vb_device_info", "vb_plan_debug_tmaps", "vb_debug_set_coverage"):
     getattr(lib, _f).restype = ctypes.c_int
 
 
@@ -233,6 +234,11 @@ def plan_from_schedule(M, N, K, lda, ldb, ldc, gemm_row, version_T, block_ptr, t
                                     int(table_id), _ptr(gr, _i32p), int(version_T), len(bp) - 1, _ptr(bp, _i32p),
                                     _ptr(tg, _i32p), _ptr(ty, _i32p), _ptr(tx, _i32p), ctypes.byref(h)))
     return Plan(h.value, batch, dtype)
+
+
+def debug_set_coverage(device: int, counts_ptr: int, c_base_ptr: int, elem_bytes: int) -> None:
+    """Coverage-counter build only (VB_LIB=.../libvbgemm_cov.so): count every stored C element."""
+    check(lib.vb_debug_set_coverage(int(device), _vp(counts_ptr), _vp(c_base_ptr), int(elem_bytes)))
 
 
 def shard_lpt(M, N, K, n_ranks: int) -> np.ndarray:

@@ -65,6 +65,16 @@ def build(force: bool = False, verbose: bool = False, trace: bool = False, defin
     return lib
 
 
+COV_LIB = os.path.join(HERE, "libvbgemm_cov.so")
+
+
+def build_coverage(force: bool = False) -> str:
+    """libvbgemm_cov.so: the same library with -DVB_COVERAGE (debug coverage counters, tests only)."""
+    if not force and os.path.exists(COV_LIB) and not _stale() and os.path.getmtime(COV_LIB) >= os.path.getmtime(LIB):
+        return COV_LIB
+    return build(defines=("VB_COVERAGE",), out="libvbgemm_cov.so")
+
+
 if __name__ == "__main__":
     defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
     outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]

@@ -39,6 +39,10 @@ cudaError_t launch_fill(int dt, int batch, const int32_t *rows, const int32_t *c
 cudaError_t launch_alpha_beta(int batch, const int64_t *gemm_id, uint64_t seed, float *alpha, float *beta,
                               cudaStream_t stream);
 cudaError_t launch_plan_expand(const ExpandArgs &a, cudaStream_t s);
+#ifdef VB_COVERAGE
+cudaError_t tc_set_coverage(int32_t *counts, const void *c_base, int es);
+cudaError_t f32_set_coverage(int32_t *counts, const void *c_base, int es);
+#endif
 cudaError_t launch_tmaps_build(const MapBuildArgs &a, cudaStream_t s);
 }  // namespace vb
 
@@ -932,6 +936,21 @@ extern "C" vb_status vb_plan_info(vb_plan_t p, int64_t *n_tiles, int64_t *n_bloc
                                            : 1 + (p->n_pair_blocks > 0) + (nb - p->n_pair_blocks > 0);  // prep + GEMMs
   }
   return VB_OK;
+}
+
+extern "C" vb_status vb_debug_set_coverage(int device, int32_t *counts, const void *c_base, int32_t elem_bytes) {
+#ifdef VB_COVERAGE
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess) return cuda_fail(g.err, "cudaSetDevice");
+  if (counts && (!c_base || (elem_bytes != 2 && elem_bytes != 4)))
+    return fail(VB_ERR_INVALID_ARG, "coverage needs the C arena base and its element size (2 or 4)");
+  cudaError_t e = tc_set_coverage(counts, c_base, elem_bytes);
+  if (e == cudaSuccess) e = f32_set_coverage(counts, c_base, elem_bytes);
+  return e == cudaSuccess ? VB_OK : cuda_fail(e, "cudaMemcpyToSymbol(coverage)");
+#else
+  (void)device; (void)counts; (void)c_base; (void)elem_bytes;
+  return fail(VB_ERR_UNSUPPORTED, "coverage counters need the -DVB_COVERAGE build (libvbgemm_cov.so)");
+#endif
 }
 
 extern "C" vb_status vb_plan_debug_tmaps(vb_plan_t p, void *out, int64_t bytes, int64_t *needed) {

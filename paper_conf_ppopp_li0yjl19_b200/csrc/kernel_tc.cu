@@ -121,7 +121,7 @@ struct Shared {
   int32_t slot_pages[kProducers][kSlots];   // per producer replica: pages charged per k-block
   int32_t acc_take[kAcc];       // MMA-private: TMEM units charged to each accumulator in flight
   uint32_t tmem_base;
-  volatile uint32_t prod_kb;    // k-blocks (>= 1 per tile) the A/B producer has finished issuing
+  uint32_t prod_kb;             // k-blocks (>= 1 per tile) the A/B producer has finished issuing (atomics only)
   TileInfo ring[kRing];
 };
 
@@ -360,7 +360,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       if (b >= p.n_blocks) break;
       int nb2 = nb;
       if (lane == 0) {
-        VB_TWAIT(T_SCHED_BUDGET, while ((int)(pushed_kb - sh->prod_kb) > kKbAhead) __nanosleep(128));
+        VB_TWAIT(T_SCHED_BUDGET, while ((int)(pushed_kb - atomicAdd(&sh->prod_kb, 0u)) > kKbAhead) __nanosleep(128));
         if (nb < p.n_blocks) nb2 = n_static + atomicAdd(p.counter, 1);   // claim two ahead
       }
       const int lim_next = (nb < p.n_blocks && lane < 2) ? p.block_ptr[nb + lane] : 0;
@@ -437,7 +437,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         advance(re, rph, kRing);
         if (ti.d.gemm < 0) break;
         if (ti.d.kblocks == 0) {
-          if (pid == 0 && leader) sh->prod_kb = sh->prod_kb + 1u;
+          if (pid == 0 && leader) atomicAdd(&sh->prod_kb, 1u);   // flow control for the scheduler
           continue;
         }
         // per-CTA geometry: a pair tile gives each CTA 128 rows of A and BX/2 columns of B
@@ -565,7 +565,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             ++ctap;
           }
           advance(slot, sph, kSlots);
-          if (pid == 0 && leader) sh->prod_kb = sh->prod_kb + 1u;
+          if (pid == 0 && leader) atomicAdd(&sh->prod_kb, 1u);   // flow control for the scheduler
         }
       }
     }
@@ -795,6 +795,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           }
           VB_TADD(T_EPI_MATH);
         }
+#ifdef VB_COVERAGE
+        if (row_ok && live && row0 + row < ti.d.M) {   // the elements this thread's row stores
+          const uint8_t *crow = static_cast<const uint8_t *>(p.C[ti.d.gemm]) + (size_t)(row0 + row) * ti.d.ldc * 2;
+          for (int j = col0 + half * hcols; j < min(col0 + (half + 1) * hcols, ti.d.N); ++j) cov_add(crow + (size_t)j * 2);
+        }
+#endif
         if ((ti.d.flags & 1) && col0 + geo.c_cols > ti.d.N) {
           // The chunk ends inside the row's last, partial 16-byte granule (N % 8 != 0): the TMA
           // store below stops at N & ~7, and the thread that computed the granule stores its
@@ -925,6 +931,10 @@ __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
 }
 
 }  // namespace tck
+
+#ifdef VB_COVERAGE
+VB_COV_SETTER(tc_set_coverage)
+#endif
 
 size_t tc_smem_bytes() { return tck::kSmemBytes; }
 

@@ -140,6 +140,28 @@ __host__ __device__ inline int tc_map_outer(int w, int M, int N, int K, int BYc)
   }
 }
 
+// Debug coverage-counter build (-DVB_COVERAGE, libvbgemm_cov.so): every element
+// an epilogue thread stores also bumps an int32 counter at the same element offset of a
+// caller-supplied counter arena (vb_debug_set_coverage), so a test can check that the tiles of
+// a plan write every C element exactly once and nothing outside the matrices.  Each kernel
+// translation unit keeps its own copy of the pointers (no relocatable device code).
+#ifdef VB_COVERAGE
+static __device__ int32_t *g_cov_counts;
+static __device__ const uint8_t *g_cov_cbase;
+static __device__ int32_t g_cov_es;
+__device__ __forceinline__ void cov_add(const void *elem) {
+  if (g_cov_counts)
+    atomicAdd(g_cov_counts + ((const uint8_t *)elem - g_cov_cbase) / g_cov_es, 1);
+}
+#define VB_COV_SETTER(name)                                                                    \
+  cudaError_t name(int32_t *counts, const void *c_base, int es) {                             \
+    cudaError_t e = cudaMemcpyToSymbol(g_cov_counts, &counts, sizeof(counts));                 \
+    if (e == cudaSuccess) e = cudaMemcpyToSymbol(g_cov_cbase, &c_base, sizeof(c_base));        \
+    if (e == cudaSuccess) e = cudaMemcpyToSymbol(g_cov_es, &es, sizeof(es));                   \
+    return e;                                                                                  \
+  }
+#endif
+
 // Tensor-core strategy geometry derived from a table row (BY, BX): TMA boxes and swizzles.
 struct TcGeom {
   int BY, BX;

@@ -52,12 +52,15 @@ constexpr TableDef kTableV100 = {1, "v100_table2", 6, VB_TABLE2_ROWS, 2, {256, 1
 // 255 registers) runs four CTAs per SM -- one warp per SMSP per CTA, so the warps that share an
 // operand ring have equal scheduler priority -- and measured 6 % faster on C2 than the
 // 256-thread version at two CTAs per SM (0.312 vs 0.332 ms), which in turn beat the full
-// 128-thread version at one CTA per SM by 13 %.  TLP threshold 4 * 148 * 256 and theta 64 from
-// the grid calibration (scripts/calibrate_grid.py); C1/C2 are insensitive to them here.
+// 128-thread version at one CTA per SM by 13 %.  TLP threshold 2 * 148 * 256 threads (= 4 tiles
+// of 128 threads per SM: one wave at four CTAs per SM) and theta 64 from the grid calibration on
+// this table (scripts/calibrate_grid.py, profiles/calibration_grid_f32_r02.json: geometric-mean
+// time over the best pair 1.042, against 1.226 for the round-1 constants calibrated on the
+// 256-thread table; theta 1 scores 1.023 but would switch K-batching off); C1/C2 are insensitive.
 constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 5,
                                      {{"small", 16, 16, 8, 1}, {"medium", 32, 32, 8, 1}, {"large", 64, 64, 8, 1},
                                       {"tall", 128, 64, 8, 1}, {"wide", 64, 128, 8, 1}},
-                                     1, {128, 0}, 4 * 148 * 256, 64, 0, 0};
+                                     1, {128, 0}, 2 * 148 * 256, 64, 0, 0};
 
 // B200 tcgen05 profile (bf16/fp16): C tiles for tcgen05.mma with M in {64,128}; BK = 64 =
 // one 128-byte swizzled row of bf16; 256 threads per tile in Eq. 1.  Besides the paper's
