@@ -23,6 +23,7 @@ class Strategy:
     BX: int      # tile columns (along N)
     BK: int      # K step of one main-loop iteration
     ctas: int = 1  # CTAs executing one tile (2 = tcgen05 cta_group::2 pair tile)
+    swap: int = 0  # 1 = swap-AB tile (C^T = B^T A^T on tcgen05; same C tile, same enumeration)
 
 
 @dataclass(frozen=True)
@@ -63,7 +64,8 @@ B200_TC = Table("b200_tcgen05", (
     Strategy("s", 64, 32, 64), Strategy("n", 128, 32, 64), Strategy("m", 64, 64, 64), Strategy("t", 128, 64, 64),
     Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("x", 64, 256, 64),
     Strategy("h", 128, 256, 64), Strategy("T2", 256, 64, 64, 2), Strategy("L2", 256, 128, 64, 2),
-    Strategy("H2", 256, 256, 64, 2)),
+    Strategy("H2", 256, 256, 64, 2), Strategy("S16", 16, 128, 64, 1, 1), Strategy("S32", 32, 128, 64, 1, 1),
+    Strategy("S48", 48, 128, 64, 1, 1), Strategy("S64", 64, 128, 64, 1, 1)),
     versions=(256,), tlp_threshold=148 * 256, theta=64)
 
 TABLES = {1: V100, 2: B200_F32, 3: B200_TC}
@@ -135,7 +137,7 @@ def b200_step1(Ms, Ns, table: Table, allow_pairs: bool) -> List[List[int]]:
     P249's rule applied to the extents of ``b200_availability`` (C-1b), over the 1-SM
     strategies only unless ``allow_pairs`` (C-7b).  Pinned by hand-derived plans in
     ``tests/golden/b200_examples.json``."""
-    order = [r for r in table.order() if allow_pairs or table.rows[r].ctas == 1]
+    order = [r for r in table.order() if (allow_pairs or table.rows[r].ctas == 1) and not table.rows[r].swap]
     queues = []
     for M, N in zip(Ms, Ns):
         mf, nf = b200_availability(M, N)

@@ -516,6 +516,7 @@ static vb_status upload(vb_plan *p, const int32_t *M, const int32_t *N, const in
     for (int r = 0; r < p->table->n_rows; ++r) {
       a.row_by[r] = (int16_t)p->table->rows[r].BY;
       a.row_bx[r] = (int16_t)p->table->rows[r].BX;
+      if (p->table->rows[r].swap) a.row_swap |= (uint16_t)(1u << r);
     }
     e = launch_plan_expand(a, s);
   }

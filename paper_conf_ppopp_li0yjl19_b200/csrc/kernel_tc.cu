@@ -169,6 +169,15 @@ __device__ __forceinline__ int acc_units(int BX, int N, int n0, bool pair) {
   const int cc = BX >= 64 ? 64 : BX;
   return ((mma_cols(BX, N, n0, pair) + cc - 1) / cc) * cc / kAccUnit;
 }
+// Swap-AB tile: the MMA's N = the tile's C rows below M, rounded up to 16 (<= BY)
+__device__ __forceinline__ int swap_rows(const TileDesc &d) {
+  return min(geo_BY(d.geo), (d.M - d.m0 + 15) & ~15);
+}
+// TMEM units (32 columns) of a tile's accumulator
+__device__ __forceinline__ int tile_acc_units(const TileDesc &d, bool pair) {
+  if (d.flags & kFlagSwap) return (swap_rows(d) + kAccUnit - 1) / kAccUnit;
+  return acc_units(geo_BX(d.geo), d.N, d.n0, pair);
+}
 // C chunks of a tile that hold any column < N (the epilogue and C producer skip the rest)
 __device__ __forceinline__ int live_chunks(const TcGeom &geo, int N, int n0) {
   const int cols = min(geo.BX, N - n0);
@@ -225,6 +234,22 @@ __device__ __forceinline__ uint32_t pack2(float lo, float hi) {
     __half2 h = __floats2half2_rn(lo, hi);
     return *reinterpret_cast<uint32_t *>(&h);
   }
+}
+
+// One C element (bf16 / fp16 bits) <-> fp32; the store rounds to nearest even (C-17).
+template <int AB_FMT>
+__device__ __forceinline__ float c_to_float(uint16_t b) {
+  if constexpr (AB_FMT == 1)
+    return __bfloat162float(__ushort_as_bfloat16(b));
+  else
+    return __half2float(__ushort_as_half(b));
+}
+template <int AB_FMT>
+__device__ __forceinline__ uint16_t float_to_c(float x) {
+  if constexpr (AB_FMT == 1)
+    return __bfloat16_as_ushort(__float2bfloat16_rn(x));
+  else
+    return __half_as_ushort(__float2half_rn(x));
 }
 
 // NU 16-byte units (8 outputs each) of this thread's row of one C chunk, starting at unit
@@ -477,7 +502,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           oy = rem / cv.Wout;
           ox = rem - oy * cv.Wout;
         }
-        const int a_pages = BY * kBK * 2 / kPageBytes;
+        const int a_pages = (BY * kBK * 2 + kPageBytes - 1) / kPageBytes;   // swap-AB tiles: 16-64 rows, 1 page
         const int need = a_pages + (Nh * kBK * 2 + kPageBytes - 1) / kPageBytes;
         for (int kb = 0; kb < ti.d.kblocks; ++kb, ++kbg) {
           int start = head, take = need;
@@ -590,7 +615,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         tr[T_TILES] += 1;
 #endif
         int take;
-        const int start = ring.place(acc_units(BX, ti.d.N, ti.d.n0, PAIR), take);
+        const int start = ring.place(tile_acc_units(ti.d, PAIR), take);
         {
           VB_T0();
           while (free_units < take || inflight == kAcc) {   // reclaim drained accumulators (FIFO)
@@ -606,9 +631,14 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         ++inflight;
         ptx::tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(start * kAccUnit);
-        const uint32_t idesc = ptx::idesc_f16((uint32_t)AB_FMT, BY, mma_cols(BX, ti.d.N, ti.d.n0, PAIR));
+        // swap-AB: A operand = the B panel (MN-major, M = BX = 128), B operand = the A rows
+        // (K-major, N = the rows below M rounded to 16); the accumulator holds C^T
+        const bool swap = (ti.d.flags & kFlagSwap) != 0;
+        const uint32_t idesc = swap ? ptx::idesc_f16_swap((uint32_t)AB_FMT, BX, swap_rows(ti.d))
+                                    : ptx::idesc_f16((uint32_t)AB_FMT, BY, mma_cols(BX, ti.d.N, ti.d.n0, PAIR));
         const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
-        const uint32_t a_bytes = (uint32_t)(PAIR ? BY / 2 : BY) * kBK * 2;
+        // B follows A's pages (whole pages: a swap-AB tile's 16-64 A rows take one)
+        const uint32_t a_bytes = (uint32_t)(((PAIR ? BY / 2 : BY) * kBK * 2 + kPageBytes - 1) / kPageBytes * kPageBytes);
         // descriptors of K step 0; step kk adds 32 B (A) / 16 rows * b_swz (B) to the start
         // address field (bits 0-13, address >> 4)
         const uint64_t adesc0 = ptx::smem_desc(0, 16, 1024, 2);
@@ -639,6 +669,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 #ifndef VB_EXP_NOMMA
               if (PAIR)
                 ptx::mma_f16_ss_pair(d_tmem, adesc + 2u * kk, bdesc + b_step * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
+              else if (swap)
+                ptx::mma_f16_ss(d_tmem, bdesc + b_step * kk, adesc + 2u * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
               else
                 ptx::mma_f16_ss(d_tmem, adesc + 2u * kk, bdesc + b_step * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
 #else
@@ -677,6 +709,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         ring_release(re);
         advance(re, rph, kRing);
         if (ti.d.gemm < 0) break;
+        if (ti.d.flags & kFlagSwap) continue;            // swap-AB tiles read C_old directly
         const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
         const TcGeom geo = tc_geom(BY, BX);
         const int row0 = ti.d.m0 + (int)rank * BY;
@@ -739,7 +772,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const uint32_t aph = (t / kAcc) & 1u;
       ++t;
       int take;
-      const int acc_col = acc_ring.place(acc_units(BX, ti.d.N, ti.d.n0, PAIR), take) * kAccUnit;
+      const int acc_col = acc_ring.place(tile_acc_units(ti.d, PAIR), take) * kAccUnit;
       // M = 128: tile row 32q + i lives in TMEM lane 32q + i.
       // M = 64 : tile row 16q + i lives in TMEM lane 32q + i, i < 16 (half sub-partitions).
       const int rows_w = BY / 4;
@@ -777,6 +810,42 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             ptx::mbar_arrive_remote(ptx::mapa(&sh->tempty[e], 0));
         }
       };
+      if (!PAIR && (ti.d.flags & kFlagSwap)) {
+        // swap-AB tile: TMEM lane 32q + i holds C column n0 + 32q + i, TMEM column j holds C row
+        // m0 + j.  Warp 8+q takes rows [0, nr/2), warp 12+q rows [nr/2, nr), eight at a time;
+        // every lane reads and writes one C column, so each row is one 64-byte warp access.
+        const int nr = swap_rows(ti.d), hr = nr / 2, j0 = half * hr;
+        const int col = ti.d.n0 + q * 32 + lane;
+        const bool col_ok = col < ti.d.N;
+        uint16_t *cc = static_cast<uint16_t *>(p.C[ti.d.gemm]) + (size_t)(ti.d.m0 + j0) * ti.d.ldc + col;
+        const int nrow = min(hr, ti.d.M - (ti.d.m0 + j0));
+        for (int jb = 0; jb < hr; jb += 8) {
+          uint32_t v[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[j] = 0u;
+          if (has_acc) {
+            ptx::tmem_ld_32x32b_x8(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc_col + j0 + jb), v);
+            ptx::tmem_ld_wait();
+          }
+          if (jb + 8 >= hr) release_acc();             // accumulator drained
+          float old[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            old[j] = (t_beta != 0.f && col_ok && jb + j < nrow) ? c_to_float<AB_FMT>(cc[(size_t)(jb + j) * ti.d.ldc])
+                                                                 : 0.f;
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            if (col_ok && jb + j < nrow) {
+              const float a = __uint_as_float(v[j]);
+              cc[(size_t)(jb + j) * ti.d.ldc] =
+                  float_to_c<AB_FMT>(t_beta != 0.f ? fmaf(t_alpha, a, t_beta * old[j]) : t_alpha * a);
+#ifdef VB_COVERAGE
+              cov_add(cc + (size_t)(jb + j) * ti.d.ldc);
+#endif
+            }
+        }
+        continue;
+      }
       auto process = [&](int ch, const uint32_t *acc) {
         const int col0 = ti.d.n0 + ch * geo.c_cols;
         VB_TWAIT(T_EPI_CFULL, ptx::mbar_wait(&sh->cfull[cs], cph));

@@ -61,6 +61,7 @@ __global__ void vb_plan_expand(ExpandArgs a) {
     }
     // the tile's last C chunk ends inside a 16-byte granule of the row: stored directly
     if ((d.N & 7) != 0 && d.n0 + BX > d.N && d.n0 < d.N) d.flags |= 1;
+    if ((a.row_swap >> r) & 1) d.flags |= kFlagSwap;
     a.tiles[k] = d;
   }
 }

@@ -80,6 +80,10 @@ struct alignas(16) ConvParam {
 };
 static_assert(sizeof(ConvParam) == 32, "ConvParam must stay 32 bytes");
 constexpr uint16_t kFlagConv = 1u << 12;
+// TileDesc.flags: swap-AB tile (C^T = B^T A^T): the MMA's A operand is the tile's B panel
+// (MN-major, M = BX = 128), its B operand the A rows (K-major, N = BY rounded to 16); the
+// accumulator holds C^T (TMEM lane = C column) and the epilogue stores it with direct stores.
+constexpr uint16_t kFlagSwap = 1u << 13;
 
 struct TcArgs {
   const int32_t *block_ptr;
@@ -106,6 +110,7 @@ struct ExpandArgs {
   TileDesc *tiles;            // tensor-core plans: TileDesc[n_slots] (else nullptr)
   TileSlot *slots;            // FFMA plans: TileSlot[n_slots] (else nullptr)
   int16_t row_by[16], row_bx[16];   // full tile extents (BY, BX) of each table row
+  uint16_t row_swap;                // bit r: table row r is a swap-AB strategy
 };
 
 // Plan-time construction of the per-GEMM tensor maps from host-encoded templates.

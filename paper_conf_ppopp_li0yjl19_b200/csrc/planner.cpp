@@ -61,12 +61,11 @@ bool pairs_allowed(const int32_t *M, const int32_t *N, const int32_t *K, int bat
 
 TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const TableDef &t,
                         int64_t threshold, bool allow_pairs) {
-  std::vector<int> order = priority_order(t);
-  if (!allow_pairs) {   // C-7b: the 1-SM version only
-    std::vector<int> o1;
-    for (int r : order)
-      if (t.rows[r].ctas == 1) o1.push_back(r);
-    order = o1;
+  std::vector<int> order;
+  for (int r : priority_order(t)) {
+    if (t.rows[r].swap) continue;                     // swap-AB rows: forced schedules only (for now)
+    if (!allow_pairs && t.rows[r].ctas != 1) continue;   // C-7b: the 1-SM version only
+    order.push_back(r);
   }
   RowCount rc[kMaxRows];
   for (int r = 0; r < t.n_rows; ++r) rc[r] = RowCount(t.rows[r]);

@@ -11,9 +11,10 @@ struct StrategyRow {
   int BX;   // C-tile columns (along N)
   int BK;   // K step of one main-loop iteration
   int ctas;   // CTAs (SMs) that execute one tile: 2 = tcgen05 cta_group::2 pair tile
+  int swap;   // 1 = swap-AB tile (tcgen05): computes C^T = B^T A^T, MMA M = BX (the N side), MMA N = BY
 };
 
-constexpr int kMaxRows = 11;
+constexpr int kMaxRows = 15;
 constexpr int kMaxVersions = 2;
 
 struct TableDef {
@@ -74,11 +75,16 @@ constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 5,
 // Constants calibrated on B200 over the Fig. 8/9 grid + C3/C4/C5 (scripts/calibrate_grid.py,
 // profiles/calibration_grid_bf16_r01.json): TLP threshold 148 * 256 (one tile per SM: the
 // persistent kernel overlaps the tiles of an SM), theta 64 (one BK = 64 k-block).
-constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 11,
+// Rows S16..S64 are swap-AB tiles for GEMMs with M <= 64 (NEXT-2): C^T = B^T A^T with the
+// MMA's M = 128 on the N side and its N = 16..64 on the M side, so a 16-row GEMM issues a
+// 128 x 16 MMA instead of a 128 x 256 one whose rows past M are discarded.
+constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 15,
                                    {{"s", 64, 32, 64, 1}, {"n", 128, 32, 64, 1}, {"m", 64, 64, 64, 1},
                                     {"t", 128, 64, 64, 1}, {"w", 64, 128, 64, 1}, {"l", 128, 128, 64, 1},
                                     {"x", 64, 256, 64, 1}, {"h", 128, 256, 64, 1},
-                                    {"T2", 256, 64, 64, 2}, {"L2", 256, 128, 64, 2}, {"H2", 256, 256, 64, 2}},
+                                    {"T2", 256, 64, 64, 2}, {"L2", 256, 128, 64, 2}, {"H2", 256, 256, 64, 2},
+                                    {"S16", 16, 128, 64, 1, 1}, {"S32", 32, 128, 64, 1, 1}, {"S48", 48, 128, 64, 1, 1},
+                                    {"S64", 64, 128, 64, 1, 1}},
                                    1, {256, 0}, 148 * 256, 64, 128, VB_TC_MIN_BX};
 
 #undef VB_TABLE2_ROWS

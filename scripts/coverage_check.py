@@ -62,6 +62,18 @@ ok &= check("pair+single/bf16", db, db.plan(0, tlp_threshold=1))
 cb = ConvBatch(vbinputs.googlenet_convs(nb=2, module="4e"), "bf16")
 cb.fill(1, "conv")
 ok &= check("conv-4e-nb2/bf16", cb, cb.plan(0))
+# every strategy row of the tcgen05 table forced (pair, 1-SM and swap-AB tiles) on ragged shapes
+from oracle import plan_ref as pr  # noqa: E402  (test infrastructure: enumerates the forced tiles)
+rows = [g % len(pr.B200_TC.rows) for g in range(len(r))]
+db = DeviceBatch(r[:, 0], r[:, 1], np.maximum(r[:, 2], 1), "bf16")
+db.fill(1)
+tl = pr.enumerate_tiles(db.M, db.N, db.K, rows, pr.B200_TC)
+pair = [pr.B200_TC.rows[rows[t.gemm]].ctas == 2 for t in tl]
+tl = [t for t, q in zip(tl, pair) if q] + [t for t, q in zip(tl, pair) if not q]
+plan = nv.plan_from_schedule(db.M, db.N, db.K, db.lda, db.ldb, db.ldc, rows, 256, list(range(len(tl) + 1)),
+                             [t.gemm for t in tl], [t.y for t in tl], [t.x for t in tl], dtype="bf16", device=0,
+                             table_id=nv.VB_TABLE_B200_TC)
+ok &= check("every-row-forced/bf16", db, plan)
 M, N, K = vbinputs.config_sizes("C4")
 db = DeviceBatch(M, N, K, "bf16")
 db.fill(1)

@@ -21,7 +21,7 @@ def test_every_c_element_written_exactly_once():
                          capture_output=True, text=True, timeout=900)
     rows = [json.loads(l) for l in out.stdout.splitlines() if l.startswith("{")]
     assert out.returncode == 0, out.stdout[-3000:] + out.stderr[-3000:]
-    assert len(rows) == 9 and all(r["wrong_counts"] == 0 and r["max_count"] == 1 for r in rows), rows
+    assert len(rows) == 10 and all(r["wrong_counts"] == 0 and r["max_count"] == 1 for r in rows), rows
 
 
 def test_product_build_rejects_coverage():

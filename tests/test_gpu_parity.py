@@ -399,3 +399,28 @@ def test_device_built_tensor_maps_equal_host_encoded(cfg, monkeypatch):
     db.run(dev_plan)
     torch.cuda.synchronize()
     check_batch(db, range(0, len(M), max(1, len(M) // 60)), SEED, "random")
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f16"])
+@pytest.mark.parametrize("ab", ["random", "conv"])
+def test_swap_ab_tiles_small_m(dtype, ab):
+    """Swap-AB strategies (S16..S64: C^T = B^T A^T, NEXT-2) forced on small-M GEMMs with N and K
+    tails, K = 0, 1-wide shapes; beta = 0 runs on NaN-poisoned C (C must not be read); elementwise
+    bound and C padding untouched."""
+    rng = np.random.default_rng(8)
+    n = 64
+    M = rng.integers(1, 65, n); N = rng.integers(1, 700, n); K = rng.integers(0, 900, n)
+    M[:4] = [1, 16, 64, 17]; N[:4] = [1, 7, 129, 256]; K[4:8] = 0
+    db = DeviceBatch(M, N, K, dtype)
+    db.C.fill_(float("nan"))
+    db.fill(SEED, ab)
+    if ab == "conv":
+        db.C.fill_(float("nan"))           # beta = 0: C_old must never be read
+    table = pr.B200_TC
+    row = {s.name: i for i, s in enumerate(table.rows)}
+    rows = [row[f"S{min(64, (int(m) + 15) // 16 * 16)}"] for m in M]
+    db.run(_forced_rows_plan(db, rows, table, 3))
+    torch.cuda.synchronize()
+    c_old = [np.zeros((int(m), int(k))) for m, k in zip(M, N)] if ab == "conv" else None
+    check_recorded(f"swapAB/{dtype}/{ab}", db, range(n), SEED, ab, c_old=c_old)
+    _padding_untouched(db)
