@@ -29,7 +29,7 @@ cudaError_t launch_f32_prep(uint8_t *tmaps, const void *const *A, const void *co
                             int batch, int32_t *counter, cudaStream_t stream);
 cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
                            const GemmParam *gemms, int batch, int32_t *counter, cudaStream_t stream);
-cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, cudaStream_t stream);
+cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, bool swap, cudaStream_t stream);
 cudaError_t tc_configure();
 cudaError_t f32_configure();
 size_t tc_smem_bytes();
@@ -109,6 +109,7 @@ struct vb_plan {
   ConvParam *d_conv = nullptr;
   int32_t *d_counter = nullptr;     // pair (FFMA) kernel [0] work-list, [1] finished CTAs; 1-SM kernel [2], [3]
   int n_pair_blocks = 0;            // blocks [0, n_pair_blocks) hold 2-SM pair tiles
+  bool has_swap = false;            // some GEMM runs a swap-AB strategy (1-SM launch with the swap path)
   int sm_count = 0;
   const void *const *bound_A = nullptr;   // last vb_plan_bind
   const void *const *bound_B = nullptr;
@@ -547,6 +548,7 @@ static vb_status finish_plan(vb_plan *p, const int32_t *M, const int32_t *N, con
   p->gemms.resize((size_t)p->batch);
   for (int i = 0; i < p->batch; ++i) {
     const StrategyRow &s = p->table->rows[p->tiling.row[i]];
+    if (s.swap && M[i] > 0 && N[i] > 0) p->has_swap = true;
     GemmParam &g = p->gemms[(size_t)i];
     g.M = M[i];
     g.N = N[i];
@@ -847,12 +849,12 @@ extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float 
     if (n_pair > 0) {
       TcArgs a{p->d_block_ptr, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter, n_pair, g_trace,
                p->d_conv};
-      e = launch_tc(a, 2 * std::min(n_pair, p->sm_count / 2), p->dt == VB_BF16, true, s);
+      e = launch_tc(a, 2 * std::min(n_pair, p->sm_count / 2), p->dt == VB_BF16, true, false, s);
     }
     if (e == cudaSuccess && n_single > 0) {
       TcArgs a{p->d_block_ptr + n_pair, p->d_tiles, p->d_tmaps, p->bound_C, alpha, beta, p->d_counter + 2, n_single,
                g_trace, p->d_conv};
-      e = launch_tc(a, std::min(n_single, p->sm_count), p->dt == VB_BF16, false, s);
+      e = launch_tc(a, std::min(n_single, p->sm_count), p->dt == VB_BF16, false, p->has_swap, s);
     }
   }
   return e == cudaSuccess ? VB_OK : cuda_fail(e, "kernel launch");

@@ -174,8 +174,8 @@ __device__ __forceinline__ int swap_rows(const TileDesc &d) {
   return min(geo_BY(d.geo), (d.M - d.m0 + 15) & ~15);
 }
 // TMEM units (32 columns) of a tile's accumulator
-__device__ __forceinline__ int tile_acc_units(const TileDesc &d, bool pair) {
-  if (d.flags & kFlagSwap) return (swap_rows(d) + kAccUnit - 1) / kAccUnit;
+__device__ __forceinline__ int tile_acc_units(const TileDesc &d, bool pair, bool swap_kernel) {
+  if (swap_kernel && (d.flags & kFlagSwap)) return (swap_rows(d) + kAccUnit - 1) / kAccUnit;
   return acc_units(geo_BX(d.geo), d.N, d.n0, pair);
 }
 // C chunks of a tile that hold any column < N (the epilogue and C producer skip the rest)
@@ -290,10 +290,12 @@ __device__ __forceinline__ void epi_row(uint8_t *cb, int row, int c_swz, int u0,
 }
 
 // --------------------------------------------------------------------------------- kernel
+// SWAP = the 1-SM variant that also runs swap-AB tiles (launched only for plans that have them,
+// so the other plans do not carry its epilogue path).
 // PAIR = the 2-SM variant (cluster of 2 CTAs, cta_group::2): every tile is a 256-row pair tile,
 // CTA r owns rows r*128.. of it and half of B; CTA 0 (the leader) schedules, issues the MMAs and
 // owns the barriers both CTAs' TMA loads and epilogues report to.
-template <int AB_FMT, bool PAIR>
+template <int AB_FMT, bool PAIR, bool SWAP = false>
 __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constant__ TcArgs p) {
   extern __shared__ uint8_t smem_raw[];
   // 1024-byte aligned (SW128 atoms); offsetting smem_raw itself keeps the shared address space
@@ -615,7 +617,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         tr[T_TILES] += 1;
 #endif
         int take;
-        const int start = ring.place(tile_acc_units(ti.d, PAIR), take);
+        const int start = ring.place(tile_acc_units(ti.d, PAIR, SWAP), take);
         {
           VB_T0();
           while (free_units < take || inflight == kAcc) {   // reclaim drained accumulators (FIFO)
@@ -633,7 +635,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const uint32_t d_tmem = tmem_base + (uint32_t)(start * kAccUnit);
         // swap-AB: A operand = the B panel (MN-major, M = BX = 128), B operand = the A rows
         // (K-major, N = the rows below M rounded to 16); the accumulator holds C^T
-        const bool swap = (ti.d.flags & kFlagSwap) != 0;
+        const bool swap = SWAP && (ti.d.flags & kFlagSwap) != 0;
         const uint32_t idesc = swap ? ptx::idesc_f16_swap((uint32_t)AB_FMT, BX, swap_rows(ti.d))
                                     : ptx::idesc_f16((uint32_t)AB_FMT, BY, mma_cols(BX, ti.d.N, ti.d.n0, PAIR));
         const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
@@ -669,7 +671,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 #ifndef VB_EXP_NOMMA
               if (PAIR)
                 ptx::mma_f16_ss_pair(d_tmem, adesc + 2u * kk, bdesc + b_step * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
-              else if (swap)
+              else if (SWAP && swap)
                 ptx::mma_f16_ss(d_tmem, bdesc + b_step * kk, adesc + 2u * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
               else
                 ptx::mma_f16_ss(d_tmem, adesc + 2u * kk, bdesc + b_step * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
@@ -709,7 +711,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         ring_release(re);
         advance(re, rph, kRing);
         if (ti.d.gemm < 0) break;
-        if (ti.d.flags & kFlagSwap) continue;            // swap-AB tiles read C_old directly
+        if (SWAP && (ti.d.flags & kFlagSwap)) continue;  // swap-AB tiles read C_old directly
         const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
         const TcGeom geo = tc_geom(BY, BX);
         const int row0 = ti.d.m0 + (int)rank * BY;
@@ -772,7 +774,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const uint32_t aph = (t / kAcc) & 1u;
       ++t;
       int take;
-      const int acc_col = acc_ring.place(tile_acc_units(ti.d, PAIR), take) * kAccUnit;
+      const int acc_col = acc_ring.place(tile_acc_units(ti.d, PAIR, SWAP), take) * kAccUnit;
       // M = 128: tile row 32q + i lives in TMEM lane 32q + i.
       // M = 64 : tile row 16q + i lives in TMEM lane 32q + i, i < 16 (half sub-partitions).
       const int rows_w = BY / 4;
@@ -810,7 +812,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             ptx::mbar_arrive_remote(ptx::mapa(&sh->tempty[e], 0));
         }
       };
-      if (!PAIR && (ti.d.flags & kFlagSwap)) {
+      if (SWAP && (ti.d.flags & kFlagSwap)) {
         // swap-AB tile: TMEM lane 32q + i holds C column n0 + 32q + i, TMEM column j holds C row
         // m0 + j.  Warp 8+q takes rows [0, nr/2), warp 12+q rows [nr/2, nr), eight at a time;
         // every lane reads and writes one C column, so each row is one 64-byte warp access.
@@ -1014,6 +1016,10 @@ cudaError_t tc_configure() {
   if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tck::vb_tc_kernel<1, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tck::vb_tc_kernel<0, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   return e;
 }
 
@@ -1025,10 +1031,14 @@ cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
 }
 
 // grid = persistent CTAs; pair = launch as clusters of 2 (grid must be even)
-cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, cudaStream_t stream) {
+cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, bool swap, cudaStream_t stream) {
   if (grid <= 0) return cudaSuccess;
   if (!pair) {
-    if (bf16)
+    if (swap && bf16)
+      tck::vb_tc_kernel<1, false, true><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
+    else if (swap)
+      tck::vb_tc_kernel<0, false, true><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
+    else if (bf16)
       tck::vb_tc_kernel<1, false><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
     else
       tck::vb_tc_kernel<0, false><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
