@@ -331,8 +331,14 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
         dist.barrier()
     torch.cuda.synchronize(dev)
     clk = clocks.stop() if clocks else None
-    step_ms = sum(s.elapsed_time(e) for s, e in zip(starts, ends)) / steps
-    kern_ms = sum(m.elapsed_time(e) for m, e in zip(mids, ends)) / steps
+    step_list = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    kern_list = [m.elapsed_time(e) for m, e in zip(mids, ends)]
+    step_ms = sum(step_list) / steps
+    kern_ms = sum(kern_list) / steps
+    pct = lambda v, q: float(np.percentile(v, q))  # noqa: E731
+    dist = {"kernel_ms_p10": pct(kern_list, 10), "kernel_ms_p50": pct(kern_list, 50),
+            "kernel_ms_p90": pct(kern_list, 90), "step_ms_p10": pct(step_list, 10),
+            "step_ms_p50": pct(step_list, 50), "step_ms_p90": pct(step_list, 90)}
     t_roof_rank = roofline_for(dtype, flops, nbytes, 1.0, peaks)["t_roof_us"]
     step_ms_max, kern_ms_max, plan_ms_max, t_roof_max = gather_max([step_ms, kern_ms, plan_ms, t_roof_rank], world,
                                                                     dist_device)
@@ -347,7 +353,13 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
         "plan": pinfo, "policy_chosen": {0: "threshold", 1: "binary", 2: "none"}.get(plan.policy(), "?"), "l2": "flushed (512 MB write) between steps" if small else
         f"inputs ({db.arena_bytes() / 1e9:.1f} GB per rank) >> L2 (126 MB); no flush",
         "launches": pinfo["launches_per_exec"] * steps, "clocks": clk, "batch_rank": int(db.batch),
+        "dist": {k: round(v, 4) for k, v in dist.items()},
     }
+    if dtype != "f32" and world == 1:
+        # compute-leaning batches (C4): the fraction also against the sustained tensor peak
+        rs = roofline_for(dtype, flops, nbytes, kern_ms * 1e-3, peaks, sustained=True)
+        res["roofline"]["frac_vs_sustained_tensor_peak"] = rs["frac"]
+        res["roofline"]["bound_vs_sustained_tensor_peak"] = rs["bound"]
     if not headline and small and world == 1:
         # the small configs also with the step (bind + exec) captured in one CUDA
         # graph and replayed (launch overhead amortised), L2 flushed outside the graph
@@ -505,11 +517,11 @@ def main_ours(args):
     if world == 1 and not args.no_aux:
         del db, plan
         torch.cuda.empty_cache()
-        for cfg in [c for c in ("C2", "C3", "C3i", "C4") if c != args.config]:
+        for cfg in [c for c in ("C1", "C2", "C3", "C3i", "C4") if c != args.config]:
             r, d2, p2 = run_config(cfg, args, world, rank, local, peaks, dist_device, headline=False)
             aux[cfg] = {"workload": workload_desc(cfg, args), "dtype": r["dtype"], "value": round(r["value"], 3),
                         "kernel_tflops": round(r["kernel_tflops"], 3), "ms_per_step": round(r["step_ms"], 4),
-                        "plan_ms": round(r["plan_ms"], 2), "roofline": _round(r["roofline"]),
+                        "plan_ms": round(r["plan_ms"], 2), "roofline": _round(r["roofline"]), "dist": r["dist"],
                         "n_tiles": r["plan"]["n_tiles"], "n_blocks": r["plan"]["n_blocks"], "l2": r["l2"],
                         "policy": r["policy_chosen"]}
             if "graph_step_ms" in r:
@@ -544,7 +556,7 @@ def main_ours(args):
             "l2": res["l2"], "plan_ms": round(res["plan_ms"], 2), "plan_first_ms": round(res["plan_first_ms"], 2),
             "n_tiles_rank0": res["plan"]["n_tiles"],
             "n_blocks_rank0": res["plan"]["n_blocks"], "kernel_ms": round(res["kernel_ms"], 4),
-            "kernel_tflops": round(res["kernel_tflops"], 3)},
+            "kernel_tflops": round(res["kernel_tflops"], 3), "timing_distribution_rank0": res["dist"]},
         "roofline": rl_out,
         "cpu_baseline": cpu,
         "e2e": res.get("e2e"),

@@ -343,6 +343,10 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     sh->prod_kb = 0u;
     ptx::fence_mbar_init();
   }
+  // pair: both CTAs' shared-memory initialisation is complete (cluster-wide) before the
+  // cta_group::2 allocation, which writes the TMEM address into shared memory asynchronously
+  // (compute-sanitizer racecheck reports the allocation against the initialisation otherwise)
+  if (PAIR) ptx::cluster_sync();
   if (warp == 1) {
     if (PAIR)
       ptx::tmem_alloc_pair(&sh->tmem_base, kTmemCols);

@@ -80,7 +80,7 @@ if __name__ == "__main__":
     tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
     os.makedirs(PROF, exist_ok=True)
     res = {}
-    for cfg in ("C5", "C4", "C2", "C3", "C3i"):
+    for cfg in ("C5", "C4", "C4single", "C2", "C3", "C3i", "C1"):
         p = os.path.join(OUT, f"prof_{cfg}.ncu-rep")
         if os.path.exists(p):
             res[cfg] = summarize(p)
@@ -91,7 +91,7 @@ if __name__ == "__main__":
         json.dump(res, f, indent=1)
     traffic = {cfg: {"dram_bytes_per_launch": int((v["dram_read_GB"] + v["dram_write_GB"]) * 1e9),
                      "source": f"profiles/ncu_{tag}.json (ncu --set full, one launch, cold)"}
-               for cfg, v in res.items() if isinstance(v, dict) and "dram_read_GB" in v}
+               for cfg, v in res.items() if isinstance(v, dict) and "dram_read_GB" in v and cfg in ("C5", "C4", "C2", "C3")}
     with open(os.path.join(PROF, "ncu_traffic.json"), "w") as f:
         json.dump(traffic, f, indent=1)
     print(json.dumps(res, indent=1))
