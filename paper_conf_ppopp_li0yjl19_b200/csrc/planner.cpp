@@ -74,10 +74,15 @@ TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const Tab
   // stored flat (no = |order| slots per GEMM, rows in priority order); pop = advance head[i],
   // top = read the head.
   const int no = (int)order.size();
+#ifdef VB_EXP_FLOOR_BY
+  const int floor_by = t.min_BY > 0 ? VB_EXP_FLOOR_BY : 0;   // experiment build: another row floor
+#else
+  const int floor_by = t.min_BY;
+#endif
   std::vector<uint8_t> q((size_t)batch * (size_t)no), qlen((size_t)batch), head((size_t)batch, 0);
   int64_t n_multi = 0;   // queues holding more than one strategy
   for (int i = 0; i < batch; ++i) {
-    const int mf = std::max<int>(M[i], t.min_BY), nf = std::max<int>(N[i], t.min_BX);   // C-1b floor
+    const int mf = std::max<int>(M[i], floor_by), nf = std::max<int>(N[i], t.min_BX);   // C-1b floor
     uint8_t *qi = &q[(size_t)i * no];
     int n = 0;
     for (int r : order)
