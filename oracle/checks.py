@@ -93,7 +93,7 @@ def check_plan_invariants(p: Plan, Ms, Ns, Ks, policy: int, theta: int) -> None:
     # tiler trace: each round's strategy per GEMM is at least as late in priority order
     # (tile area never shrinks).  Which strategies were available (P249, or the B200 pre-pass)
     # is pinned by hand-derived plans in tests/golden, not re-derived here.
-    tr = p.tiling.trace
+    tr = p.tiling.trace[:-1] if p.tiling.filled else p.tiling.trace   # the fill round shrinks tiles (C-1d)
     pos = {r: i for i, r in enumerate(p.table.order())}
     for (r0, _, _), (r1, _, _) in zip(tr, tr[1:]):
         assert all(pos[b] >= pos[a] for a, b in zip(r0, r1))

@@ -88,6 +88,7 @@ class TilingResult:
     rows: List[int]            # chosen table row per GEMM
     T: int                     # chosen version (threads per block)
     trace: List[Tuple[List[int], int, int]] = field(default_factory=list)  # (rows, T, TLP) per round
+    filled: bool = False       # the last trace entry is the TLP fill post-pass (reading C-1d)
 
     def ids(self, table: Table) -> List[int]:
         return [table.strategy_id(r, self.T) for r in self.rows]
@@ -179,6 +180,54 @@ def tiling_engine(Ms, Ns, table: Table, threshold: int | None = None,
                 T = table.versions[vi]
             elif single_before:
                 return TilingResult(cur, T, trace)
+
+
+def tlp_fill(Ms, Ns, Ks, table: Table, threshold: int, tr: TilingResult) -> TilingResult:
+    """Reading C-1d, the B200 tcgen05 post-pass on the tiling engine's solution.  When the
+    final round's TLP is within the threshold (the wave is not full): take the GEMMs whose
+    tiles carry the most operand bytes, K * (min(BY, M) + min(BX, N)); if every one of them can split its tiles
+    -- the strategy with the same BY and half the BX (same CTA count) if that gives it more
+    tiles, else the one with the same BX and half the BY -- and the TLP with all of them moved
+    stays <= threshold, move them all and repeat; otherwise stop.  The filled
+    TLP is appended to the trace when some GEMM moved."""
+    rows, T = list(tr.rows), tr.T
+    t = tr.trace[-1][2]
+    if t > threshold:
+        return tr
+
+    def tiles(g, r):
+        s = table.rows[r]
+        return ceil(Ms[g] / s.BY) * ceil(Ns[g] / s.BX) * s.ctas
+
+    def split(g):
+        """Half the width (same BY) if that gives GEMM g more tiles, else half the height."""
+        s = table.rows[rows[g]]
+        for same_by in (True, False):
+            for q, x in enumerate(table.rows):
+                if x.ctas != s.ctas or x.swap != s.swap:
+                    continue
+                fits = (x.BY == s.BY and 2 * x.BX == s.BX) if same_by else (x.BX == s.BX and 2 * x.BY == s.BY)
+                if fits and tiles(g, q) > tiles(g, rows[g]):
+                    return q
+        return None
+
+    live = [g for g in range(len(rows)) if Ms[g] > 0 and Ns[g] > 0 and Ks[g] > 0]
+    moved = False
+    while live:
+        work = {g: Ks[g] * (min(table.rows[rows[g]].BY, Ms[g]) + min(table.rows[rows[g]].BX, Ns[g])) for g in live}
+        top = [g for g in live if work[g] == max(work.values())]
+        targets = [split(g) for g in top]
+        if any(h is None for h in targets):
+            break
+        add = sum(tiles(g, h) - tiles(g, rows[g]) for g, h in zip(top, targets))
+        if t + add * T > threshold:
+            break
+        for g, h in zip(top, targets):
+            rows[g] = h
+        t += add * T
+        moved = True
+    trace = tr.trace + ([(list(rows), T, t)] if moved else [])
+    return TilingResult(rows, T, trace, moved)
 
 
 # ----------------------------------------------------------------------------------------
@@ -331,6 +380,8 @@ def plan(Ms, Ns, Ks, table: Table, policy: int = POLICY_THRESHOLD,
     else:
         q = step1_p249(Ms, Ns, table)
     tr = tiling_engine(Ms, Ns, table, thr, q)
+    if table is B200_TC:
+        tr = tlp_fill(Ms, Ns, Ks, table, thr, tr)
     all_tiles = enumerate_tiles(Ms, Ns, Ks, tr.rows, table)
     is_pair = [table.rows[tr.rows[t.gemm]].ctas == 2 for t in all_tiles]
     tiles = [t for t, pp in zip(all_tiles, is_pair) if pp] + [t for t, pp in zip(all_tiles, is_pair) if not pp]

@@ -607,6 +607,7 @@ static vb_status plan_impl(int device, vb_dtype dt, int32_t batch, const int32_t
   PhaseClock clk;
   p->tiling = tiling_engine(M, N, batch, *t, thr, !conv && pairs_allowed(M, N, K, batch, elem_bytes(dt)));
   if (batch == 0) p->tiling.version_T = t->versions[0];
+  if (t->min_BY > 0) tlp_fill(M, N, K, batch, *t, thr, p->tiling);   // the tcgen05 table's post-pass (C-1d)
   clk.mark("tiling engine");
   p->seg = build_segments(M, N, batch, p->tiling.row, *t);
   clk.mark("enumeration");

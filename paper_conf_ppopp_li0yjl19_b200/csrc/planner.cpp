@@ -129,6 +129,62 @@ TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const Tab
   }
 }
 
+void tlp_fill(const int32_t *M, const int32_t *N, const int32_t *K, int batch, const TableDef &t, int64_t threshold,
+              TilingOut &out) {
+  // Reading C-1d (B200 tcgen05 table): the tiling engine stops at the first round whose TLP is
+  // within the threshold, all GEMMs moving together.  When that round leaves TLP below the
+  // threshold (the SMs of one wave are not all used), the spare TLP goes to the critical path:
+  // the GEMMs whose tiles carry the most operand bytes (K * (min(BY, M) + min(BX, N))) all split their tiles --
+  // half the width (same BY) if that gives the GEMM more tiles, else half the height (same BX)
+  // -- only if every one of them can and the TLP stays within the threshold; the step repeats
+  // on the new maximum.
+  if (out.trace.empty() || out.trace.back().tlp > threshold) return;
+  const int T = out.version_T;
+  int64_t tlp = out.trace.back().tlp;
+  bool moved = false;
+  auto tiles = [&](int g, int r) { return cdiv(M[g], t.rows[r].BY) * cdiv(N[g], t.rows[r].BX) * t.rows[r].ctas; };
+  // the strategy a GEMM's tiles split into: half the width if that gives the GEMM more tiles,
+  // else half the height; -1 if neither exists or adds tiles
+  auto half_of = [&](int g) {
+    const StrategyRow &s = t.rows[out.row[(size_t)g]];
+    for (int dim = 0; dim < 2; ++dim)
+      for (int q = 0; q < t.n_rows; ++q) {
+        const StrategyRow &c = t.rows[q];
+        if (c.ctas != s.ctas || c.swap != s.swap) continue;
+        const bool fits = dim == 0 ? (c.BY == s.BY && 2 * c.BX == s.BX) : (c.BX == s.BX && 2 * c.BY == s.BY);
+        if (fits && tiles(g, q) > tiles(g, out.row[(size_t)g])) return q;
+      }
+    return -1;
+  };
+  auto work = [&](int g) {   // operand bytes per k-block of the GEMM's (interior) tile, ~ K (BY + BX)
+    const StrategyRow &s = t.rows[out.row[(size_t)g]];
+    return (int64_t)K[g] * (std::min<int64_t>(s.BY, M[g]) + std::min<int64_t>(s.BX, N[g]));
+  };
+  for (;;) {
+    int64_t wmax = -1;
+    for (int g = 0; g < batch; ++g)
+      if (M[g] > 0 && N[g] > 0 && K[g] > 0) wmax = std::max(wmax, work(g));
+    if (wmax <= 0) break;
+    int64_t add = 0;
+    bool ok = true;
+    for (int g = 0; g < batch && ok; ++g) {
+      if (M[g] <= 0 || N[g] <= 0 || K[g] <= 0 || work(g) != wmax) continue;
+      const int h = half_of(g);
+      if (h < 0) ok = false;
+      else add += tiles(g, h) - tiles(g, out.row[(size_t)g]);
+    }
+    if (!ok || tlp + add * (int64_t)T > threshold) break;
+    std::vector<int> target((size_t)batch, -1);
+    for (int g = 0; g < batch; ++g)
+      if (M[g] > 0 && N[g] > 0 && K[g] > 0 && work(g) == wmax) target[(size_t)g] = half_of(g);
+    for (int g = 0; g < batch; ++g)
+      if (target[(size_t)g] >= 0) out.row[(size_t)g] = target[(size_t)g];
+    tlp += add * (int64_t)T;
+    moved = true;
+  }
+  if (moved) out.trace.push_back({tlp, T});   // the filled plan's TLP, reported as one more round
+}
+
 Segments build_segments(const int32_t *M, const int32_t *N, int batch, const std::vector<int> &row,
                         const TableDef &t) {
   // Tile enumeration (P133-135, P157, P284) in compact form: GEMM g with strategy (BY, BX)

@@ -49,6 +49,11 @@ int64_t tlp_eq1(const int32_t *M, const int32_t *N, int batch, const std::vector
 TilingOut tiling_engine(const int32_t *M, const int32_t *N, int batch, const TableDef &t,
                         int64_t threshold, bool pairs_allowed = true);
 
+// Reading C-1d (B200 tcgen05 table): after the tiling engine, spend TLP left below the threshold
+// on the longest-K GEMMs by halving their tile width (one more trace entry when it applies).
+void tlp_fill(const int32_t *M, const int32_t *N, const int32_t *K, int batch, const TableDef &t, int64_t threshold,
+              TilingOut &out);
+
 // Reading C-7b: offer the 2-SM pair strategies only to batches with arithmetic intensity
 // 2*sum(MNK) / sum(es*(MK+KN) + 2*es*MN) >= 128 flop/byte.
 bool pairs_allowed(const int32_t *M, const int32_t *N, const int32_t *K, int batch, int elem_bytes);

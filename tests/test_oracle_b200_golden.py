@@ -109,3 +109,16 @@ def test_kworkload_floor(g):
     assert [len(b) for b in pr.threshold_batching(tiles, 256, 0, 64)] == e["zero_block_sizes"]
     tiles = [pr.Tile(0, i, 0, k) for i, k in enumerate(e["mixed_K"])]
     assert [len(b) for b in pr.threshold_batching(tiles, 256, 0, 64)] == e["mixed_block_sizes"]
+
+
+def test_tlp_fill_post_pass(g):
+    e = g["E2_tlp_fill"]
+    M, N, K = [list(c) for c in zip(*e["gemms_MNK"])]
+    assert pr.pairs_allowed(M, N, K) is False
+    tr = pr.tiling_engine(M, N, TC, e["threshold"], pr.b200_step1(M, N, TC, False))
+    assert _names(tr.rows) == e["tiler_final"]
+    filled = pr.tlp_fill(M, N, K, TC, e["threshold"], tr)
+    assert _names(filled.rows) == e["final"] and filled.trace[-1][2] == e["final_tlp"]
+    assert len(filled.trace) == e["rounds"]
+    p = pr.plan(M, N, K, TC, pr.POLICY_THRESHOLD, tlp_threshold=e["threshold"])
+    assert _names(p.tiling.rows) == e["final"]
