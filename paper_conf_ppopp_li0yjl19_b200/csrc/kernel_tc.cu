@@ -966,11 +966,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   // bound plan -- including replays of a CUDA graph that captured only vb_exec_bound -- need no
   // reset.  Every CTA made its final claim (one that returned >= n_blocks) before getting here.
   if (threadIdx.x == 0) {
-    __threadfence();
-    if (atomicAdd(&p.counter[1], 1) == (int)gridDim.x - 1) {
+    if (ptx::atom_add_acq_rel_gpu(&p.counter[1], 1) == (int)gridDim.x - 1) {
       atomicExch(&p.counter[0], 0);
       atomicExch(&p.counter[1], 0);
-      __threadfence();
     }
     VB_STAMP(10);
   }
