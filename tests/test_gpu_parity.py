@@ -424,3 +424,23 @@ def test_swap_ab_tiles_small_m(dtype, ab):
     c_old = [np.zeros((int(m), int(k))) for m, k in zip(M, N)] if ab == "conv" else None
     check_recorded(f"swapAB/{dtype}/{ab}", db, range(n), SEED, ab, c_old=c_old)
     _padding_untouched(db)
+
+
+def test_replanning_loop_reuses_workspaces_and_stays_exact():
+    """The paper's on-line case (P272): sizes vary per call and every call plans again.  Forty
+    plans of varying batches (bf16 and fp32) are built, executed and destroyed in turn (the
+    workspaces cycle through the per-device pool); every result is checked."""
+    rng = np.random.default_rng(31)
+    for it in range(40):
+        dtype = "bf16" if it % 3 else "f32"
+        n = int(rng.integers(1, 40))
+        M, N, K = (rng.integers(1, 400, n) for _ in range(3))
+        db = DeviceBatch(M, N, K, dtype)
+        db.C.fill_(float("nan"))
+        db.fill(it)
+        plan = db.plan(vb.VB_BATCH_AUTO)
+        db.run(plan)
+        torch.cuda.synchronize()
+        check_batch(db, range(n), it, "random")
+        _padding_untouched(db)
+        del plan, db
