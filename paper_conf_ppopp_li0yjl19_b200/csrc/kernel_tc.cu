@@ -99,6 +99,17 @@ static_assert(sizeof(TileInfo) == 48, "TileInfo size");
 // done, 2 first ring entry pushed, 3 first k-block armed by a producer, 4 MMA saw its first
 // k-block, 5 first accumulator committed, 6 epilogue saw it, 7 epilogue done with it, 8 its
 // stores complete, 9 teardown barrier passed, 10 exit.
+#ifdef VB_TIMELINE_ALL
+// Opt-in (measurement only): every CTA stores %globaltimer at entry and exit into
+// p.trace[2 * blockIdx.x + {0, 1}] (the buffer holds 2 * gridDim.x entries).
+__device__ __forceinline__ void vb_stamp_all(long long *buf, int i) {
+  if (buf) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    buf[2 * blockIdx.x + i] = (long long)t;
+  }
+}
+#endif
 #ifdef VB_TIMELINE
 __device__ __forceinline__ void vb_stamp(long long *buf, int i) {
   if (blockIdx.x == 0 && buf) {
@@ -302,6 +313,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   // visible to the compiler, so C-slot and barrier accesses compile to LDS/STS, not generic LD/ST.
   uint8_t *smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   if (threadIdx.x == 0) VB_STAMP(0);
+#ifdef VB_TIMELINE_ALL
+  if (threadIdx.x == 0) vb_stamp_all(p.trace, 0);
+#endif
   uint8_t *pages = smem;
   uint8_t *cbuf = smem + (size_t)kPages * kPageBytes;
   Shared *sh = reinterpret_cast<Shared *>(cbuf + (size_t)kCSlots * kCSlotBytes);
@@ -971,6 +985,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       atomicExch(&p.counter[1], 0);
     }
     VB_STAMP(10);
+#ifdef VB_TIMELINE_ALL
+    vb_stamp_all(p.trace, 1);
+#endif
   }
 }
 
