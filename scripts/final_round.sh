@@ -9,7 +9,7 @@ VB_PARITY_OUT=$OUT/parity_final.json timeout 1200 python -m pytest tests -m gpu 
 tail -2 $OUT/gputest_final.log
 VB_SAN_TIMEOUT=420 bash scripts/sanitize.sh $OUT/sanitizer_final > /dev/null 2>&1
 cat $OUT/sanitizer_final/summary.txt
-VB_LIB=paper_conf_ppopp_li0yjl19_b200/libvbgemm_cov.so timeout 900 python scripts/coverage_check.py > $OUT/coverage_final.jsonl 2>&1
+VB_LIB=paper_conf_ppopp_li0yjl19_b200/libvbgemm_cov.so timeout 900 python tests/tools/coverage_check.py > $OUT/coverage_final.jsonl 2>&1
 tail -3 $OUT/coverage_final.jsonl
 bash scripts/profile_round.sh > $OUT/profile_round.log 2>&1
 tail -c 300 $OUT/bench_default.json

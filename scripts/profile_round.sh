@@ -17,5 +17,5 @@ timeout 600 $NCU -k regex:vb_tc_kernel -o $OUT/prof_C3i -f python scripts/prof_k
 timeout 600 $NCU -k regex:vb_tc_kernel -o $OUT/prof_C3 -f python scripts/prof_kernel.py --config C3 > $OUT/prof_C3.log 2>&1
 timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none --csv python bench.py --steps 3 --warmup 3 --e2e-steps 1 --cpu-seconds 2 > $OUT/launches_c5.csv 2> $OUT/launches_c5.err
 timeout 1200 python bench.py > $OUT/bench_default.json 2> $OUT/bench_default.err
-timeout 600 python scripts/oracle_timing.py > $OUT/oracle_timing.jsonl 2>&1
+timeout 600 python tests/tools/oracle_timing.py > $OUT/oracle_timing.jsonl 2>&1
 tail -c 400 $OUT/bench_default.json

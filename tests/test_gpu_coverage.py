@@ -1,5 +1,5 @@
 """Debug coverage-counter build: every C element is stored by exactly one tile,
-nothing outside the matrices is stored.  Runs scripts/coverage_check.py in a subprocess with the
+nothing outside the matrices is stored.  Runs tests/tools/coverage_check.py in a subprocess with the
 -DVB_COVERAGE library (libvbgemm_cov.so, built by __graft_entry__.build())."""
 import json
 import os
@@ -17,7 +17,7 @@ def test_every_c_element_written_exactly_once():
     import build as vbbuild
     lib = vbbuild.build_coverage()
     env = dict(os.environ, VB_LIB=lib)
-    out = subprocess.run([sys.executable, os.path.join(ROOT, "scripts", "coverage_check.py")], env=env, cwd=ROOT,
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "tests", "tools", "coverage_check.py")], env=env, cwd=ROOT,
                          capture_output=True, text=True, timeout=900)
     rows = [json.loads(l) for l in out.stdout.splitlines() if l.startswith("{")]
     assert out.returncode == 0, out.stdout[-3000:] + out.stderr[-3000:]

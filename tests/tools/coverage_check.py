@@ -1,7 +1,7 @@
 """Coverage-counter check (SURVEY.md §4 GPU row: "debug coverage-counter build: each C element
 written exactly once").  Run with the -DVB_COVERAGE library:
 
-    VB_LIB=paper_conf_ppopp_li0yjl19_b200/libvbgemm_cov.so python scripts/coverage_check.py
+    VB_LIB=paper_conf_ppopp_li0yjl19_b200/libvbgemm_cov.so python tests/tools/coverage_check.py
 
 For each batch (both policies): zero an int32 counter per element of the C arena, run
 vb_exec_vbatched, and require counter == 1 on every element of every C matrix and 0 everywhere
@@ -13,7 +13,7 @@ import json
 import os
 import sys
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 assert "libvbgemm_cov" in os.environ.get("VB_LIB", ""), "run with VB_LIB=.../libvbgemm_cov.so"
 

@@ -6,7 +6,7 @@ import os
 import sys
 import time
 
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
 import vbinputs  # noqa: E402
 from oracle import plan_ref as pr  # noqa: E402
 import paper_conf_ppopp_li0yjl19_b200 as vb  # noqa: E402

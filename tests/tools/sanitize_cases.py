@@ -2,7 +2,7 @@
 through the C-ABI and checks the result against the fp64 oracle, so a sanitizer run also
 proves the instrumented kernels still compute the right thing.
 
-    compute-sanitizer --tool memcheck python scripts/sanitize_cases.py [case ...]
+    compute-sanitizer --tool memcheck python tests/tools/sanitize_cases.py [case ...]
 
 cases: c1 (C1 fp32, 3 policies), ragged_bf16 / ragged_f32 (48 GEMMs, M, N, K in [1, 600]),
 pair (2-SM cta_group::2 tiles + 1-SM tiles, two GEMM launches), conv (GoogleNet 3a implicit
@@ -11,7 +11,7 @@ GEMM, TMA im2col), graph (vb_exec_bound captured in a CUDA graph, 3 replays).
 import os
 import sys
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 sys.path.insert(0, os.path.join(ROOT, "tests"))
 

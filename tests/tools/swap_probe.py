@@ -1,13 +1,13 @@
 """Swap-AB tiles (S16..S64) against the 128x256 tile for the GEMMs with M <= 64 of a batch,
 through forced schedules (vb_plan_from_schedule, one tile per block, enumeration order).
 
-    python scripts/swap_probe.py [C5|C3|small]
+    python tests/tools/swap_probe.py [C5|C3|small]
 """
 import os
 import sys
 
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
+sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))), "tests"))
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
