@@ -373,6 +373,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   else
     __syncthreads();
   ptx::tc_fence_after();
+#ifndef VB_NO_PDL
+  // programmatic dependent launch: the setup above overlapped the bind-time prep kernel; the
+  // tensor maps it patches and the work-list counters it resets are used only after this wait
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+#endif
   const uint32_t tmem_base = sh->tmem_base;
   if (threadIdx.x == 0) VB_STAMP(1);
   const uint8_t *tmaps = reinterpret_cast<const uint8_t *>(p.tmaps);
@@ -999,6 +1004,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 // buffers to check that no stale descriptor is ever used.
 __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *const *B, void *const *C,
                            const GemmParam *gemms, int batch, int32_t *counter) {
+#ifndef VB_NO_PDL
+  asm volatile("griddepcontrol.launch_dependents;");   // the GEMM kernel may start its setup now
+#endif
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i == 0) {
     counter[0] = counter[1] = 0;   // pair kernel
@@ -1052,31 +1060,37 @@ cudaError_t launch_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
 // grid = persistent CTAs; pair = launch as clusters of 2 (grid must be even)
 cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, bool swap, cudaStream_t stream) {
   if (grid <= 0) return cudaSuccess;
-  if (!pair) {
-    if (swap && bf16)
-      tck::vb_tc_kernel<1, false, true><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
-    else if (swap)
-      tck::vb_tc_kernel<0, false, true><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
-    else if (bf16)
-      tck::vb_tc_kernel<1, false><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
-    else
-      tck::vb_tc_kernel<0, false><<<grid, tck::kThreads, tck::kSmemBytes, stream>>>(args);
-    return cudaGetLastError();
-  }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3(tck::kThreads);
   cfg.dynamicSmemBytes = tck::kSmemBytes;
   cfg.stream = stream;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = 2;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
+  cudaLaunchAttribute attr[2];
+  int na = 0;
+#ifndef VB_NO_PDL
+  // programmatic dependent launch: may start while the previous kernel on the stream (the
+  // bind-time prep kernel) finishes; the kernel waits for it (griddepcontrol.wait) after setup
+  attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[na].val.programmaticStreamSerializationAllowed = 1;
+  ++na;
+#endif
+  if (pair) {
+    attr[na].id = cudaLaunchAttributeClusterDimension;
+    attr[na].val.clusterDim.x = 2;
+    attr[na].val.clusterDim.y = 1;
+    attr[na].val.clusterDim.z = 1;
+    ++na;
+  }
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
-  return bf16 ? cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<1, true>, args)
-              : cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<0, true>, args);
+  cfg.numAttrs = (unsigned)na;
+  if (pair)
+    return bf16 ? cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<1, true>, args)
+                : cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<0, true>, args);
+  if (swap)
+    return bf16 ? cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<1, false, true>, args)
+                : cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<0, false, true>, args);
+  return bf16 ? cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<1, false>, args)
+              : cudaLaunchKernelEx(&cfg, tck::vb_tc_kernel<0, false>, args);
 }
 
 }  // namespace vb
