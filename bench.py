@@ -11,9 +11,10 @@ at 1/2/4/8 B200; % of roofline").
   collective on the data path; NCCL only for the barrier and the timing gather).
   The total batch is fixed as N grows -> "scaling": "strong".
 * step = one vb_exec_vbatched over the rank's shard with inputs resident in HBM:
-  the bind-time prep kernel (tensor-map addresses) + the persistent GEMM kernel, launched
-  programmatically behind it.  The kernel-only time for the roofline comes from a second pass
-  of K steps with an event between the two launches.
+  vb_plan_bind (tensor-map prep kernel) + vb_exec_bound (the persistent GEMM kernel), with a
+  CUDA event between the two that gives the GEMM kernel's own duration for the roofline (the
+  event also keeps the GEMM kernel from starting its setup under the prep kernel, as its
+  programmatic launch does in a plain vb_exec_vbatched call -- see cuda_graph_step_ms and e2e).
   Planning (tiling + batching engines, descriptor upload) happens once per batch shape and is
   reported separately as plan_ms.  The inputs (30.5 GB) are far larger than L2 (126 MB).
 * value = sum over ranks of 2*M*N*K / max over ranks of the timed region (CUDA events on the
@@ -298,10 +299,7 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
     flush = torch.empty(int(512e6), dtype=torch.uint8, device=dev) if small else None
     stream = torch.cuda.current_stream(dev)
 
-    def step():                                    # one vb_exec_vbatched: bind (prep) + GEMM kernel(s)
-        db.run(plan, stream)
-
-    def kernel_step():                             # the same, with an event between bind and the GEMM kernel
+    def step():
         db.bind(plan, stream)
         ev_mid = torch.cuda.Event(enable_timing=True)
         ev_mid.record(stream)
@@ -320,32 +318,16 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
     if clocks:
         clocks.start()
         time.sleep(0.3)
-    # the timed region: K steps of the public call.  (An event between bind and the GEMM kernel
-    # would serialise the GEMM kernel's programmatic launch behind the prep kernel, so the
-    # kernel-only time is taken in a second pass of K steps below.)
-    starts, ends = [], []
+    starts, mids, ends = [], [], []
     for _ in range(steps):
         if flush is not None:
             flush.fill_(1)                          # evict L2 between timed iterations
         s = torch.cuda.Event(enable_timing=True)
         s.record(stream)
-        step()
+        m = step()
         e = torch.cuda.Event(enable_timing=True)
         e.record(stream)
-        starts.append(s); ends.append(e)
-    torch.cuda.synchronize(dev)
-    if world > 1:
-        import torch.distributed as dist
-        dist.barrier()
-    torch.cuda.synchronize(dev)
-    mids, kends = [], []
-    for _ in range(steps):                         # kernel-only pass (roofline): GEMM launch(es) alone
-        if flush is not None:
-            flush.fill_(1)
-        m = kernel_step()
-        e = torch.cuda.Event(enable_timing=True)
-        e.record(stream)
-        mids.append(m); kends.append(e)
+        starts.append(s); mids.append(m); ends.append(e)
     torch.cuda.synchronize(dev)
     if world > 1:
         import torch.distributed as dist
@@ -353,7 +335,7 @@ def run_config(cfg, args, world, rank, local, peaks, dist_device, headline=True)
     torch.cuda.synchronize(dev)
     clk = clocks.stop() if clocks else None
     step_list = [s.elapsed_time(e) for s, e in zip(starts, ends)]
-    kern_list = [m.elapsed_time(e) for m, e in zip(mids, kends)]
+    kern_list = [m.elapsed_time(e) for m, e in zip(mids, ends)]
     step_ms = sum(step_list) / steps
     kern_ms = sum(kern_list) / steps
     pct = lambda v, q: float(np.percentile(v, q))  # noqa: E731
