@@ -96,7 +96,11 @@ typedef struct vb_plan *vb_plan_t;
  *           (else VB_ERR_ALIGNMENT).
  *  policy   batching policy.   tuning: nullable (all defaults).
  *  out      receives the plan.  The plan owns its device descriptors and workspace.
- * Device plans copy their descriptors to the device synchronously before returning.
+ * Device plans upload the compact schedule (Tile[], slot order, GEMM segments, per-GEMM
+ * parameters, tensor-map templates) in one copy on a private stream, expand it on the device
+ * into per-slot tile records and per-GEMM tensor maps, and synchronise that stream before
+ * returning.  The workspace comes from a per-device stream-ordered memory pool that keeps
+ * freed memory for the next plan (VB_NO_PLAN_POOL=1 in the environment: plain cudaMalloc).
  * ------------------------------------------------------------------------------------ */
 vb_status vb_plan_vbatched(int device, vb_dtype dt, int32_t batch,
                            const int32_t *M, const int32_t *N, const int32_t *K,
@@ -166,7 +170,9 @@ vb_status vb_plan_conv(int device, vb_dtype dt, int32_t batch, const vb_conv_des
  * Never allocates, never synchronises.  Enqueues at most three kernels: the descriptor
  * prep kernel (tensor-map address patch and work-counter reset), then the GEMM kernel(s) --
  * fp32: one FFMA kernel; bf16/fp16: the 2-SM pair kernel (if the plan has pair tiles) and
- * the 1-SM kernel.  All of it may be captured in a CUDA graph.  The caller
+ * the 1-SM kernel.  The GEMM kernels are launched with programmatic stream serialisation
+ * (they start their setup while the prep kernel runs and wait for it before touching its
+ * output).  All of it may be captured in a CUDA graph.  The caller
  * keeps every buffer alive until the stream work completes.  A plan may be re-executed
  * with new pointers / alpha / beta, but not concurrently on two streams.
  * Returns VB_ERR_CUDA if a launch fails (vb_last_error() has the CUDA message).
