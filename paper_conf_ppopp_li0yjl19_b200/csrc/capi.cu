@@ -2,6 +2,7 @@
 // tensor-map encoding, exec dispatch, export of the device plan, input fill.
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 #include <cudaTypedefs.h>
 #include <stdarg.h>
 #include <stdlib.h>
@@ -64,6 +65,12 @@ static vb_status fail(vb_status s, const char *fmt, ...) {
   g_last_error = buf;
   return s;
 }
+// NVTX range for profilers (header-only NVTX 3: no cost unless a tool is attached)
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+
 // VB_PLAN_PROFILE=1: planning phase times on stderr (host clock; measurement aid only)
 struct PhaseClock {
   bool on = getenv("VB_PLAN_PROFILE") != nullptr;
@@ -604,6 +611,7 @@ static vb_status plan_impl(int device, vb_dtype dt, int32_t batch, const int32_t
     }
   }
   PhaseClock clk;
+  NvtxRange nvtx_plan("vb_plan (tiling + batching engines, descriptors)");
   p->tiling = tiling_engine(M, N, batch, *t, thr, !conv && pairs_allowed(M, N, K, batch, elem_bytes(dt)));
   if (batch == 0) p->tiling.version_T = t->versions[0];
   if (t->min_BY > 0) tlp_fill(M, N, K, batch, *t, thr, p->tiling);   // the tcgen05 table's post-pass (C-1d)
@@ -806,6 +814,7 @@ struct DeviceGuard {
 
 extern "C" vb_status vb_plan_bind(vb_plan_t p, const void *const *A, const void *const *B, void *const *C,
                                   void *stream) {
+  NvtxRange nvtx("vb_plan_bind");
   if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
   if (p->device < 0) return fail(VB_ERR_UNSUPPORTED, "host-only plan cannot be executed");
   if (p->batch > 0 && (!A || !B || !C)) return fail(VB_ERR_INVALID_ARG, "null pointer array");
@@ -826,6 +835,7 @@ extern "C" vb_status vb_plan_bind(vb_plan_t p, const void *const *A, const void 
 }
 
 extern "C" vb_status vb_exec_bound(vb_plan_t p, const float *alpha, const float *beta, void *stream) {
+  NvtxRange nvtx("vb_exec_bound");
   if (!p) return fail(VB_ERR_INVALID_ARG, "plan is null");
   if (p->device < 0) return fail(VB_ERR_UNSUPPORTED, "host-only plan cannot be executed");
   if (p->batch == 0) return VB_OK;
