@@ -56,6 +56,12 @@ constexpr int kPageBytes = 8192;
 #ifndef VB_KB_PREFETCH
 #define VB_KB_PREFETCH 0   // experiment: L2 prefetch of each A/B box this many k-blocks ahead
 #endif
+#ifndef VB_A_NEXT_PREFETCH
+#define VB_A_NEXT_PREFETCH 0   // experiment: L2 prefetch of the next k-block's A box at even k-blocks
+#endif
+#ifndef VB_C_NEXT_PREFETCH
+#define VB_C_NEXT_PREFETCH 0   // experiment: L2 prefetch of the next C_old chunk at even chunks
+#endif
 #ifndef VB_A_PAIR_PREFETCH
 #define VB_A_PAIR_PREFETCH 0   // experiment: L2 prefetch of the A box 2 k-blocks ahead at even k-blocks
 #endif
@@ -598,6 +604,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             // promotion DRAM sees 512 contiguous bytes of each A row requested together
             if (i == 0 && (kb & 1) == 0 && kb + 2 < ti.d.kblocks) ptx::tma_prefetch_2d(mapA, (kb + 2) * kBK, row0);
 #endif
+#if VB_A_NEXT_PREFETCH
+            // even k-blocks: L2-prefetch the next k-block's A box right behind this one, so DRAM
+            // sees 256 contiguous bytes of each A row requested together (a 128-byte box alone
+            // streams at ~4.9 TB/s, two adjacent ones at ~7.3 TB/s: profiles/tma_locality_r01.txt)
+            if (i == 0 && (kb & 1) == 0 && kb + 1 < ti.d.kblocks) ptx::tma_prefetch_2d(mapA, (kb + 1) * kBK, row0);
+#endif
 #if VB_KB_PREFETCH > 0
             // start the DRAM fetch of the same box VB_KB_PREFETCH k-blocks ahead into L2
             if (kb + VB_KB_PREFETCH < ti.d.kblocks) {
@@ -757,6 +769,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
               ptx::tma_load_2d(cbuf + (size_t)cs * kCSlotBytes + w * rows_w * geo.c_swz, mapC, &sh->cfull[cs],
                                ti.d.n0 + ch * geo.c_cols, row0 + w * rows_w);
 #endif
+#if VB_C_NEXT_PREFETCH
+            // even chunks: L2-prefetch the next chunk's sub-boxes (the adjacent 128 bytes of each row)
+            if ((ch & 1) == 0 && ch + 1 < nch)
+              for (int w = 2 * cid; w < 2 * cid + nsub; ++w)
+                ptx::tma_prefetch_2d(mapC, ti.d.n0 + (ch + 1) * geo.c_cols, row0 + w * rows_w);
+#endif
           } else {
             ptx::mbar_arrive(&sh->cfull[cs]);
           }
@@ -792,7 +810,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const TcGeom geo = tc_geom(BY, BX);
       const int row0 = ti.d.m0 + (int)rank * BY;     // this CTA's first row of the tile
       const uint8_t *mapC = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128) + MAP_C_ST * 128;
+#ifdef VB_EXP_C_RMW
+      const int n8 = (ti.d.N + 7) & ~7;
+#else
       const int n8 = ti.d.N & ~7;                       // the store map's width
+#endif
       const int e = (int)(t % kAcc);
       const uint32_t aph = (t / kAcc) & 1u;
       ++t;
@@ -895,7 +917,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           for (int j = col0 + half * hcols; j < min(col0 + (half + 1) * hcols, ti.d.N); ++j) cov_add(crow + (size_t)j * 2);
         }
 #endif
+#if defined(VB_EXP_NOSTORE) || defined(VB_EXP_NOTAIL)
+        if (false) {
+#else
         if ((ti.d.flags & 1) && col0 + geo.c_cols > ti.d.N) {
+#endif
           // The chunk ends inside the row's last, partial 16-byte granule (N % 8 != 0): the TMA
           // store below stops at N & ~7, and the thread that computed the granule stores its
           // N % 8 elements itself.
@@ -903,10 +929,17 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           const int grow = row0 + row;
           if (g0 >= half * hcols && g0 < (half + 1) * hcols && row_ok && grow < ti.d.M) {
             const uint4 w = *reinterpret_cast<const uint4 *>(cb + ptx::swz((uint32_t)(row * geo.c_swz + g0 * 2), geo.c_swz));
-            const uint16_t *h = reinterpret_cast<const uint16_t *>(&w);
-            uint16_t *crow = reinterpret_cast<uint16_t *>(static_cast<uint8_t *>(p.C[ti.d.gemm]) +
-                                                          ((size_t)grow * ti.d.ldc + n8) * 2);
-            for (int j = 0; j < (ti.d.N & 7); ++j) crow[j] = h[j];
+            uint8_t *crow = static_cast<uint8_t *>(p.C[ti.d.gemm]) + ((size_t)grow * ti.d.ldc + n8) * 2;
+            // the granule is 16-byte aligned: its N % 8 elements go out as at most three stores
+            // (8 + 4 + 2 bytes) -- one L2 write per store and row, not one per element
+            const int nt = ti.d.N & 7;
+            if (nt & 4) *reinterpret_cast<uint2 *>(crow) = make_uint2(w.x, w.y);
+            if (nt & 2) *reinterpret_cast<uint32_t *>(crow + (nt & 4) * 2) = (nt & 4) ? w.z : w.x;
+            if (nt & 1) {
+              const int e = nt & 6;                       // the last element's index in the granule
+              const uint32_t word = e >= 4 ? (e == 6 ? w.w : w.z) : (e == 2 ? w.y : w.x);
+              *reinterpret_cast<uint16_t *>(crow + e * 2) = (uint16_t)(word & 0xFFFFu);
+            }
           }
         }
         // TMA store of the quarter's sub-box; rows >= M and columns >= N & ~7 are clipped by the

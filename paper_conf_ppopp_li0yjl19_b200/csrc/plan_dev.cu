@@ -86,7 +86,12 @@ __global__ void vb_tmaps_build(MapBuildArgs a) {
   uint8_t *m = a.tmaps + (size_t)i * 128;
   const bool is_a = w <= 1, is_b = w == 2 || w == 3;
   const uint64_t es = (uint64_t)a.es;
+#ifdef VB_EXP_C_RMW
+  // experiment (timing only): C_old loaded and C stored through whole 16-byte granules
+  const uint32_t inner = is_a ? gp.K : is_b ? gp.N : (uint32_t)((gp.N + 7) & ~7);
+#else
   const uint32_t inner = is_a ? gp.K : is_b ? gp.N : w == MAP_C ? gp.N : (gp.N & ~7);
+#endif
   const uint32_t rows = is_a ? gp.M : is_b ? gp.K : gp.M;
   const uint64_t stride = (uint64_t)(is_a ? gp.lda : is_b ? gp.ldb : gp.ldc) * es;
   const int c = outer ? a.tidx[tmap_key(w, gp.row & 0xFF, outer, (rows - 1) * stride + inner * es < kTmapSmallBytes)]

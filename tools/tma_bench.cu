@@ -39,6 +39,7 @@ __global__ void __launch_bounds__(256, 1) tma_stream(const __grid_constant__ CUt
     int st = 0;
     uint32_t ph = 0;
     unsigned t = blockIdx.x * 7919u + pid * 104729u;
+    int pair_next = 0;
     for (int it = 0; it < a.iters / P; ++it) {
       const int s = pid * per + st;
       ptx::mbar_wait(&empty[s], ph ^ 1u);
@@ -51,6 +52,20 @@ __global__ void __launch_bounds__(256, 1) tma_stream(const __grid_constant__ CUt
           const int groups_w = tiles_w / a.boxes_per_stage;
           const int g = (int)(t % (unsigned)(groups_w * tiles_h));
           tile = (g / groups_w) * tiles_w + (g % groups_w) * a.boxes_per_stage + b;
+        } else if (a.sequential >= 3) {      // pairs of adjacent boxes in consecutive stages
+          if ((it & 1) == 0) {
+            t = t * 1664525u + 1013904223u;
+            const int groups_w = tiles_w / 2;
+            const int g = (int)(t % (unsigned)(groups_w * tiles_h));
+            tile = (g / groups_w) * tiles_w + (g % groups_w) * 2;
+            if (a.sequential == 3) {          // 3: L2-prefetch the adjacent box with this one
+              const int tx = ((tile + 1) % tiles_w) * a.box_w, ty = ((tile + 1) / tiles_w) * a.box_h;
+              ptx::tma_prefetch_2d(&map, tx, ty);
+            }
+            pair_next = tile + 1;
+          } else {
+            tile = pair_next;                 // 4: the adjacent box one stage later, no prefetch
+          }
         } else { t = t * 1664525u + 1013904223u; tile = (int)(t % (unsigned)ntiles); }
         const int x = (tile % tiles_w) * a.box_w, y = (tile / tiles_w) * a.box_h;
         ptx::tma_load_2d(smem + (size_t)s * a.stage_bytes + (size_t)b * a.box_w * a.box_h * 2, &map, &full[s], x, y);
@@ -90,7 +105,10 @@ int main(int argc, char **argv) {
   cudaMalloc(&buf, (size_t)rows * cols * 2);
   cudaMemset(buf, 0, (size_t)rows * cols * 2);
   CUtensorMap map;
-  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  // TMA_INNER < cols: the map's row length is shorter than the stride, so the last box of each
+  // row is partly out of bounds (zero-filled), like the K tail of an A matrix
+  const int inner = getenv("TMA_INNER") ? atoi(getenv("TMA_INNER")) : cols;
+  cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)rows};
   cuuint64_t strides[1] = {(cuuint64_t)cols * 2};
   cuuint32_t box[2] = {(cuuint32_t)box_w, (cuuint32_t)box_h};
   cuuint32_t es[2] = {1, 1};
@@ -98,7 +116,7 @@ int main(int argc, char **argv) {
   CUtensorMapSwizzle swz = sw == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : sw == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
                                                                              : CU_TENSOR_MAP_SWIZZLE_32B;
   CUresult r = cuTensorMapEncodeTiled(&map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, buf, dims, strides, box, es,
-                                      CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                      CU_TENSOR_MAP_INTERLEAVE_NONE, swz, getenv("TMA_PROMO") ? (CUtensorMapL2promotion)atoi(getenv("TMA_PROMO")) : CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     printf("encode failed %d\n", (int)r);
