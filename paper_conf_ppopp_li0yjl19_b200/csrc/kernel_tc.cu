@@ -56,6 +56,9 @@ constexpr int kPageBytes = 8192;
 #ifndef VB_KB_PREFETCH
 #define VB_KB_PREFETCH 0   // experiment: L2 prefetch of each A/B box this many k-blocks ahead
 #endif
+#ifndef VB_EPI_FFMA2
+#define VB_EPI_FFMA2 1   // epilogue alpha*acc + beta*C_old as paired fp32 FMUL2/FFMA2 (0: scalar)
+#endif
 #ifndef VB_A_NEXT_PREFETCH
 #define VB_A_NEXT_PREFETCH 0   // experiment: L2 prefetch of the next k-block's A box at even k-blocks
 #endif
@@ -286,8 +289,20 @@ __device__ __forceinline__ void epi_row(uint8_t *cb, int row, int c_swz, int u0,
     for (int u = 0; u < NU; ++u) {
       float old[8], o[8];
       unpack8<AB_FMT>(w[u], old);
+#if VB_EPI_FFMA2
+      // paired fp32 ops (FMUL2 / FFMA2): the same two roundings per element as the scalar form
+#pragma unroll
+      for (int e = 0; e < 8; e += 2) {
+        const float2 bo = __fmul2_rn(make_float2(beta, beta), make_float2(old[e], old[e + 1]));
+        const float2 r = __ffma2_rn(make_float2(alpha, alpha),
+                                    make_float2(__uint_as_float(acc[u * 8 + e]), __uint_as_float(acc[u * 8 + e + 1])), bo);
+        o[e] = r.x;
+        o[e + 1] = r.y;
+      }
+#else
 #pragma unroll
       for (int e = 0; e < 8; ++e) o[e] = fmaf(alpha, __uint_as_float(acc[u * 8 + e]), beta * old[e]);
+#endif
       w[u].x = pack2<AB_FMT>(o[0], o[1]);
       w[u].y = pack2<AB_FMT>(o[2], o[3]);
       w[u].z = pack2<AB_FMT>(o[4], o[5]);
