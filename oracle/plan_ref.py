@@ -57,7 +57,7 @@ B200_F32 = Table("b200_ffma", V100.rows[:5], versions=(128,), tlp_threshold=2 * 
 
 # B200 tcgen05 (bf16/fp16) profile: C-tile shapes sized for tcgen05.mma
 # (M in {64,128}), BK = 64 (one 128-byte swizzle row of bf16), plus the skinny shapes
-# 128x32 and 64x256, plus 2-SM pair tiles 256x{64,128,256} (ctas = 2, cta_group::2).  One
+# 128x32 and 64x256, plus 2-SM pair tiles 256x{64,128,256,512} (ctas = 2, cta_group::2).  One
 # kernel "version" with T = 256 threads.  Its step 1 is the B200 pre-pass
 # ``b200_step1`` below (readings C-1b, C-7b), not P249's literal rule.
 B200_TC = Table("b200_tcgen05", (
@@ -65,7 +65,7 @@ B200_TC = Table("b200_tcgen05", (
     Strategy("w", 64, 128, 64), Strategy("l", 128, 128, 64), Strategy("x", 64, 256, 64),
     Strategy("h", 128, 256, 64), Strategy("T2", 256, 64, 64, 2), Strategy("L2", 256, 128, 64, 2),
     Strategy("H2", 256, 256, 64, 2), Strategy("S16", 16, 128, 64, 1, 1), Strategy("S32", 32, 128, 64, 1, 1),
-    Strategy("S48", 48, 128, 64, 1, 1), Strategy("S64", 64, 128, 64, 1, 1)),
+    Strategy("S48", 48, 128, 64, 1, 1), Strategy("S64", 64, 128, 64, 1, 1), Strategy("W2", 256, 512, 64, 2)),
     versions=(256,), tlp_threshold=148 * 256, theta=64)
 
 TABLES = {1: V100, 2: B200_F32, 3: B200_TC}

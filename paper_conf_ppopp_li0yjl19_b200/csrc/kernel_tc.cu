@@ -182,6 +182,12 @@ __device__ __forceinline__ int mma_cols(int BX, int N, int n0, bool pair) {
   const int cols = min(BX, N - n0);
   return min(BX, (cols + g - 1) & ~(g - 1));
 }
+// MMA N of half h of a tile whose MMA width is mc: a W2 pair tile (BX = 512) issues two MMAs
+// per K step, half h covering the tile's columns [256h, 256h + width) into TMEM columns
+// [256h, ..); every other tile has one half (mc <= 256).
+__device__ __forceinline__ int half_cols(int mc, int h) { return h == 0 ? min(mc, 256) : max(0, mc - 256); }
+// shared-memory bytes between the two halves' B panels of one CTA (128 columns x BK rows)
+constexpr int kHalfBBytes = 128 * 64 * 2;
 // TMEM columns (32-column units) an accumulator occupies: its MMA width rounded up to whole
 // epilogue chunks (the epilogue reads every column of a live chunk), not BX, so tiles at the
 // right edge of narrow GEMMs leave room for more accumulators in flight
@@ -213,7 +219,9 @@ struct AccRing {
     int start = head;
     take = units;
     if (start + units > kAccUnits) {
-      take += kAccUnits - start;
+      // charge the skipped end of the ring too; a 512-column accumulator (W2) overlaps it, and
+      // the charge is the union of the two regions (the whole ring)
+      take += kAccUnits - start - max(0, units - start);
       start = 0;
     }
     head = start + units;
@@ -513,9 +521,11 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         }
         // per-CTA geometry: a pair tile gives each CTA 128 rows of A and BX/2 columns of B
         const int BY = geo_BY(ti.d.geo) / (PAIR ? 2 : 1), BX = geo_BX(ti.d.geo);
-        const int BXc = PAIR ? BX / 2 : BX;
+        const int BXc = PAIR ? min(BX, 256) / 2 : BX;   // B columns of one MMA half in this CTA
         const TcGeom geo = tc_geom(BY, BXc);
-        const int Nh = mma_cols(BX, ti.d.N, ti.d.n0, PAIR) / (PAIR ? 2 : 1);   // B columns per CTA
+        // MMA halves (two for a W2 tile): half h's B columns per CTA (a pair splits each evenly)
+        const int mc = mma_cols(BX, ti.d.N, ti.d.n0, PAIR);
+        const int Nh0 = half_cols(mc, 0) / (PAIR ? 2 : 1), Nh1 = half_cols(mc, 1) / (PAIR ? 2 : 1);
         const uint8_t *maps = tmaps + (size_t)ti.d.gemm * (kMapsPerGemm * 128);
         // out-of-bounds box rows cost L2 bandwidth even though TMA zero-fills them: the last
         // row-tile uses the row-tail map, the last k-block the K-tail map, and B boxes that lie
@@ -525,15 +535,18 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           const int rows = min(BY, ti.d.M - (ti.d.m0 + r * BY));
           return rows <= 0 ? 0 : (rows < BY ? (rows + 7) / 8 * 8 : BY);
         };
-        auto b_boxes_of = [&](int r) {
-          const int cols = min(Nh, ti.d.N - (ti.d.n0 + r * Nh));
+        auto b_boxes_half = [&](int r, int h) {
+          const int nh = h ? Nh1 : Nh0;
+          const int cols = min(nh, ti.d.N - (ti.d.n0 + h * 256 + r * nh));
           const int bw = geo.b_swz / 2;                  // a power of two: shift, not divide
           return cols <= 0 ? 0 : min(geo.b_boxes, (cols + bw - 1) >> (__ffs(bw) - 1));
         };
-        const int row0 = ti.d.m0 + (int)rank * BY, col0 = ti.d.n0 + (int)rank * Nh;
+        auto b_boxes_of = [&](int r) { return b_boxes_half(r, 0) + (Nh1 ? b_boxes_half(r, 1) : 0); };
+        const int row0 = ti.d.m0 + (int)rank * BY;
         const int a_box_rows = a_box_rows_of((int)rank);
         const bool a_tail = a_box_rows != BY;
         const uint8_t *mapA = maps + (a_tail ? MAP_A_TAIL : MAP_A) * 128;
+        const int b_boxes0 = b_boxes_half((int)rank, 0);
         const int b_boxes = b_boxes_of((int)rank);
         const int ksteps_last = (ti.d.flags >> 8) & 7;
         // implicit GEMM (vb_plan_conv): the window origin of this CTA's first output pixel
@@ -549,7 +562,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           ox = rem - oy * cv.Wout;
         }
         const int a_pages = (BY * kBK * 2 + kPageBytes - 1) / kPageBytes;   // swap-AB tiles: 16-64 rows, 1 page
-        const int need = a_pages + (Nh * kBK * 2 + kPageBytes - 1) / kPageBytes;
+        const int b_span = Nh1 ? kHalfBBytes + Nh1 * kBK * 2 : Nh0 * kBK * 2;   // B panel bytes of this CTA
+        const int need = a_pages + (b_span + kPageBytes - 1) / kPageBytes;
         for (int kb = 0; kb < ti.d.kblocks; ++kb, ++kbg) {
           int start = head, take = need;
           if (start + need > kPages) {          // never wrap a k-block around the ring end
@@ -591,7 +605,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           if (ptx::elect_lane0())
           for (int i = (int)((pid - kbg) % kProducers + kProducers) % kProducers; i <= b_boxes; i += kProducers) {
             if (i == 0 && a_box_rows == 0) continue;
-            uint8_t *dst = i == 0 ? sa : sb + (i - 1) * kBK * geo.b_swz;
+            // B box i - 1: box j of half h (half 1 at kHalfBBytes, columns 256 on)
+            const int h = i - 1 >= b_boxes0 ? 1 : 0, j = i - 1 - h * b_boxes0;
+            uint8_t *dst = i == 0 ? sa : sb + h * kHalfBBytes + j * kBK * geo.b_swz;
             const uint8_t *map = i == 0 ? mapA : mapB;
             if (conv) {   // k-block kb = (tap ctap, channel block ccb)
               if (i == 0) {
@@ -599,12 +615,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
                 ptx::tma_load_im2col_4d(dst, map, &sh->full[slot], ccb * kBK, ox - cv.pad, oy - cv.pad, img,
                                         (uint16_t)kw, (uint16_t)kh);
               } else {
-                ptx::tma_load_2d(dst, map, &sh->full[slot], col0 + (i - 1) * (geo.b_swz / 2),
+                ptx::tma_load_2d(dst, map, &sh->full[slot], ti.d.n0 + (int)rank * Nh0 + j * (geo.b_swz / 2),
                                  ctap * cv.Cin + ccb * kBK);
               }
               continue;
             }
-            const int c0 = i == 0 ? kb * kBK : col0 + (i - 1) * (geo.b_swz / 2);
+            const int c0 = i == 0 ? kb * kBK : ti.d.n0 + h * 256 + (int)rank * (h ? Nh1 : Nh0) + j * (geo.b_swz / 2);
             const int c1 = i == 0 ? row0 : kb * kBK;
             if (PAIR)
               ptx::tma_load_2d_pair(dst, map, &sh->full[slot], c0, c1);
@@ -660,7 +676,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         advance(re, rph, kRing);
         if (ti.d.gemm < 0) break;
         const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);   // MMA shape (pair: M = 256)
-        const TcGeom geo = tc_geom(PAIR ? BY / 2 : BY, PAIR ? BX / 2 : BX);   // this CTA's B half
+        const TcGeom geo = tc_geom(PAIR ? BY / 2 : BY, PAIR ? min(BX, 256) / 2 : BX);   // this CTA's B half
         const int e = (int)(t % kAcc);
         ++t;
 #ifdef VB_TRACE
@@ -686,8 +702,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         // swap-AB: A operand = the B panel (MN-major, M = BX = 128), B operand = the A rows
         // (K-major, N = the rows below M rounded to 16); the accumulator holds C^T
         const bool swap = SWAP && (ti.d.flags & kFlagSwap) != 0;
+        const int mc = mma_cols(BX, ti.d.N, ti.d.n0, PAIR);
         const uint32_t idesc = swap ? ptx::idesc_f16_swap((uint32_t)AB_FMT, BX, swap_rows(ti.d))
-                                    : ptx::idesc_f16((uint32_t)AB_FMT, BY, mma_cols(BX, ti.d.N, ti.d.n0, PAIR));
+                                    : ptx::idesc_f16((uint32_t)AB_FMT, BY, half_cols(mc, 0));
+        // W2 pair tile: the second MMA half (columns 256.., B panel at kHalfBBytes, TMEM +256)
+        const int mc1 = PAIR ? half_cols(mc, 1) : 0;
+        const uint32_t idesc1 = mc1 ? ptx::idesc_f16((uint32_t)AB_FMT, BY, mc1) : 0u;
         const uint32_t blayout = ptx::swizzle_layout_code(geo.b_swz);
         // B follows A's pages (whole pages: a swap-AB tile's 16-64 A rows take one)
         const uint32_t a_bytes = (uint32_t)(((PAIR ? BY / 2 : BY) * kBK * 2 + kPageBytes - 1) / kPageBytes * kPageBytes);
@@ -719,9 +739,12 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
             for (int kk = 0; kk < kBK / 16; ++kk) {
               if (kk >= ksteps) break;          // K tail: the B rows past the last step are not loaded
 #ifndef VB_EXP_NOMMA
-              if (PAIR)
+              if (PAIR) {
                 ptx::mma_f16_ss_pair(d_tmem, adesc + 2u * kk, bdesc + b_step * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
-              else if (SWAP && swap)
+                if (mc1)
+                  ptx::mma_f16_ss_pair(d_tmem + 256u, adesc + 2u * kk, bdesc + (uint32_t)(kHalfBBytes >> 4) + b_step * kk,
+                                       idesc1, (kb | kk) != 0 ? 1u : 0u);
+              } else if (SWAP && swap)
                 ptx::mma_f16_ss(d_tmem, bdesc + b_step * kk, adesc + 2u * kk, idesc, (kb | kk) != 0 ? 1u : 0u);
               else
                 ptx::mma_f16_ss(d_tmem, adesc + 2u * kk, bdesc + b_step * kk, idesc, (kb | kk) != 0 ? 1u : 0u);

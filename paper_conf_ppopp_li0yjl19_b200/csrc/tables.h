@@ -14,7 +14,7 @@ struct StrategyRow {
   int swap;   // 1 = swap-AB tile (tcgen05): computes C^T = B^T A^T, MMA M = BX (the N side), MMA N = BY
 };
 
-constexpr int kMaxRows = 15;
+constexpr int kMaxRows = 16;
 constexpr int kMaxVersions = 2;
 
 struct TableDef {
@@ -78,13 +78,18 @@ constexpr TableDef kTableB200Ffma = {2, "b200_ffma", 5,
 // Rows S16..S64 are swap-AB tiles for GEMMs with M <= 64 (NEXT-2): C^T = B^T A^T with the
 // MMA's M = 128 on the N side and its N = 16..64 on the M side, so a 16-row GEMM issues a
 // 128 x 16 MMA instead of a 128 x 256 one whose rows past M are discarded.
-constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 15,
+// Row W2 (256 x 512, 2-SM) is the widest pair tile: each SM holds 128 rows of A and two
+// 128-column halves of B and issues two N = 256 MMAs per K step into all 512 TMEM columns, so a
+// k-block carries twice the MMA work of H2 for 1.5x its bytes (the latency its operand ring
+// covers grows by 1.5x at equal shared memory) -- the shape cuBLAS's own heuristic runs for
+// large bf16 GEMMs on B200 (nvjet_tst_256x256_64x4_2x1_2cta: 256 x 256 C elements per CTA).
+constexpr TableDef kTableB200Tc = {3, "b200_tcgen05", 16,
                                    {{"s", 64, 32, 64, 1}, {"n", 128, 32, 64, 1}, {"m", 64, 64, 64, 1},
                                     {"t", 128, 64, 64, 1}, {"w", 64, 128, 64, 1}, {"l", 128, 128, 64, 1},
                                     {"x", 64, 256, 64, 1}, {"h", 128, 256, 64, 1},
                                     {"T2", 256, 64, 64, 2}, {"L2", 256, 128, 64, 2}, {"H2", 256, 256, 64, 2},
                                     {"S16", 16, 128, 64, 1, 1}, {"S32", 32, 128, 64, 1, 1}, {"S48", 48, 128, 64, 1, 1},
-                                    {"S64", 64, 128, 64, 1, 1}},
+                                    {"S64", 64, 128, 64, 1, 1}, {"W2", 256, 512, 64, 2}},
                                    1, {256, 0}, 148 * 256, 64, 128, VB_TC_MIN_BX};
 
 #undef VB_TABLE2_ROWS

@@ -41,6 +41,10 @@ cases = {
 for b, m, n, k in [(4096, 128, 256, 1024), (16384, 256, 256, 256), (16384, 200, 200, 200),
                    (65536, 128, 256, 128), (65536, 100, 100, 100), (65536, 64, 64, 64)]:
     cases[f"u{b}x{m}x{n}x{k}"] = (np.full(b, m), np.full(b, n), np.full(b, k))
+# compute-bound uniform batches (tensor-pipe feed of the pair kernel; cuBLAS context in
+# scripts/cublas_context.py)
+for b, m, n, k in [(64, 1024, 1024, 4096), (16, 2048, 2048, 4096), (256, 512, 512, 2048)]:
+    cases[f"c{b}x{m}x{n}x{k}"] = (np.full(b, m), np.full(b, n), np.full(b, k))
 for k in (16, 32, 40, 48, 56, 64, 72, 100, 128, 200, 256):
     cases[f"K{k}"] = (np.full(32768, 128), np.full(32768, 256), np.full(32768, k))
 for n in (16, 17, 20, 24, 25, 29, 31, 32, 33, 40, 48, 64, 100, 128, 200, 256):
@@ -69,6 +73,7 @@ for name in only:
     nbytes = 2 * ((M * K).sum() + (K * N).sum() + mn * (1 if loads_only else 2))
     print(json.dumps(dict(case=name, lib=os.path.basename(os.environ.get("VB_LIB", "libvbgemm.so")), ms=round(ms, 4),
                           GB=round(nbytes / 1e9, 2), TBps=round(nbytes / ms / 1e9, 3),
+                          TFLOPs=round(2 * (M * N * K).sum() / ms / 1e9, 1),
                           tiles=plan.info()["n_tiles"])), flush=True)
     del db, plan
     torch.cuda.empty_cache()

@@ -288,6 +288,27 @@ def test_pair_tiles_selected_for_compute_bound_batch(dtype):
     _padding_untouched(db)
 
 
+@pytest.mark.parametrize("dtype", ["bf16", "f16"])
+def test_w2_tiles_forced(dtype):
+    """W2 (256 x 512 pair tile: two N <= 256 MMAs per K step into 512 TMEM columns) forced on
+    every GEMM: N tails inside the first half (N - n0 <= 256: one MMA), inside the second half
+    (the pair splits each half evenly, CTA 1's share of half 1 possibly empty), row tails on
+    either CTA, K tails and K = 0, beta != 0; alternating with H2 so that 512-column and
+    256-column accumulators share the TMEM ring."""
+    N = np.array([512, 300, 260, 289, 511, 513, 700, 1000, 1024, 257, 33, 640, 768, 520])
+    M = np.array([256, 300, 129, 512, 255, 100, 384, 777, 1024, 256, 256, 130, 17, 600])
+    K = np.array([64, 100, 4096, 0, 1000, 63, 1500, 17, 2048, 640, 128, 300, 700, 1])
+    db = DeviceBatch(M, N, K, dtype)
+    db.C.fill_(float("nan"))
+    db.fill(SEED)
+    rows = [15 if g % 3 else 10 for g in range(len(M))]
+    db.run(_forced_rows_plan(db, rows, pr.B200_TC, 3))
+    torch.cuda.synchronize()
+    check_batch(db, range(len(M)), SEED, "random")
+    check_bound(db, range(len(M)), SEED, "random")
+    _padding_untouched(db)
+
+
 # ------------------------------------------------------------------ policy selection (P272-274)
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])
 def test_auto_policy_parity(dtype):
