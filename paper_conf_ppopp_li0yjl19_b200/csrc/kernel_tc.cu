@@ -243,13 +243,15 @@ __device__ __forceinline__ void unpack8(uint4 w, float (&f)[8]) {
   const uint32_t u[4] = {w.x, w.y, w.z, w.w};
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
-    float2 v;
-    if constexpr (AB_FMT == 1)
-      v = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162 *>(&u[i]));
-    else
-      v = __half22float2(*reinterpret_cast<const __half2 *>(&u[i]));
-    f[2 * i] = v.x;
-    f[2 * i + 1] = v.y;
+    if constexpr (AB_FMT == 1) {
+      // bf16 -> fp32 is exact and is the bf16 bits in the top half: one SHL / LOP3 each
+      f[2 * i] = __uint_as_float(u[i] << 16);
+      f[2 * i + 1] = __uint_as_float(u[i] & 0xFFFF0000u);
+    } else {
+      const float2 v = __half22float2(*reinterpret_cast<const __half2 *>(&u[i]));
+      f[2 * i] = v.x;
+      f[2 * i + 1] = v.y;
+    }
   }
 }
 
