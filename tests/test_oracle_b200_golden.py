@@ -6,7 +6,9 @@ out next to it):
   contrasted with P249's literal step 1 on the same GEMMs;
 * the pair-version gate ``pairs_allowed`` (C-7b) on both sides of 128 flop/B;
 * the per-launch batching of pair and 1-SM tiles (C-7b launch split) under both heuristics;
-* the K-workload floor of threshold batching (C-11).
+* the K-workload floor of threshold batching (C-11);
+* the W2 pair row (256 x 512): its availability and its place at the end of the priority order
+  (E3), in the oracle and in the product planner.
 """
 import json
 import os
@@ -122,3 +124,31 @@ def test_tlp_fill_post_pass(g):
     assert len(filled.trace) == e["rounds"]
     p = pr.plan(M, N, K, TC, pr.POLICY_THRESHOLD, tlp_threshold=e["threshold"])
     assert _names(p.tiling.rows) == e["final"]
+
+
+def test_w2_row_availability_and_priority(g):
+    e = g["E3_w2"]
+    M, N, K = [list(c) for c in zip(*e["gemms_MNK"])]
+    assert pr.pairs_allowed(M, N, K) is e["pairs_allowed"]
+    assert TC.rows[e["w2_table_row"]].name == "W2"
+    q = pr.b200_step1(M, N, TC, allow_pairs=True)
+    assert [_names(x) for x in q] == e["b200_queues"]
+    tr = pr.tiling_engine(M, N, TC, 5000, q)
+    assert [[_names(r), t] for r, _, t in tr.trace] == [[a, b] for a, b in e["rounds"]]
+    assert _names(tr.rows) == e["final_thr5000"]
+    tr = pr.tiling_engine(M, N, TC, 5632, pr.b200_step1(M, N, TC, allow_pairs=True))
+    assert _names(tr.rows) == e["final_thr5632"]
+
+
+@pytest.mark.parametrize("thr,key", [(5000, "final_thr5000"), (5632, "final_thr5632")])
+def test_w2_row_product_planner(g, thr, key):
+    """The C++ tiling engine picks the same rows as the hand derivation (host plan, no GPU)."""
+    import numpy as np
+    import paper_conf_ppopp_li0yjl19_b200 as vb
+    e = g["E3_w2"]
+    M, N, K = (np.array(c) for c in zip(*e["gemms_MNK"]))
+    ld = (N + 7) // 8 * 8                     # 16-byte rows
+    p = vb.plan_vbatched(M, N, K, K, ld, ld, "bf16", vb.VB_BATCH_THRESHOLD, device=-1,
+                         table_id=vb.VB_TABLE_B200_TC, tlp_threshold=thr)
+    rows = [int(s) % len(TC.rows) for s in p.export()["gemm_strategy"]]
+    assert _names(rows) == e[key]
