@@ -994,7 +994,10 @@ extern "C" vb_status vb_plan_export(vb_plan_t p, int32_t *block_ptr, int32_t *ti
       e = cudaMemcpy(td.data(), p->d_tiles, td.size() * sizeof(TileDesc), cudaMemcpyDeviceToHost);
       for (size_t k = 0; k < td.size() && e == cudaSuccess; ++k) {
         const int BY = (td[k].geo & 0xFF) * 16, BX = (td[k].geo >> 8) * 16;
-        sl[k] = TileSlot{(uint32_t)td[k].gemm, (uint16_t)(td[k].m0 / BY), (uint16_t)(td[k].n0 / BX)};
+        const int Ng = p->gemms[(size_t)td[k].gemm].N;
+        const bool swp = p->table->rows[p->gemms[(size_t)td[k].gemm].row & 0xFF].swap != 0;
+        sl[k] = TileSlot{(uint32_t)td[k].gemm, (uint16_t)(td[k].m0 / BY),
+                         (uint16_t)(swp ? td[k].n0 / BX : tile_col_index(td[k].n0, Ng, BX))};
       }
     } else if (e == cudaSuccess && !sl.empty()) {
       e = cudaMemcpy(sl.data(), p->d_slots, sl.size() * sizeof(TileSlot), cudaMemcpyDeviceToHost);

@@ -43,10 +43,14 @@ __global__ void vb_plan_expand(ExpandArgs a) {
     TileDesc d;
     d.gemm = g;
     d.m0 = y * BY;
-    d.n0 = x * BX;
     d.kblocks = gp.kblocks;
     d.M = gp.M;
-    d.N = gp.N;
+    if ((a.row_swap >> r) & 1) {   // swap-AB tiles keep the fixed split (their epilogue tests N per column)
+      d.n0 = x * BX;
+      d.N = gp.N;
+    } else {
+      tile_cols(x, gp.N, BX, d.n0, d.N);
+    }
     d.ldc = gp.ldc;
     d.geo = (uint16_t)((BY / 16) | ((BX / 16) << 8));
     d.flags = 0;
@@ -60,7 +64,8 @@ __global__ void vb_plan_expand(ExpandArgs a) {
       d.flags |= (uint16_t)(((gp.K % 64 + 15) / 16) << 8);   // MMA K-steps of the last k-block
     }
     // the tile's last C chunk ends inside a 16-byte granule of the row: stored directly
-    if ((d.N & 7) != 0 && d.n0 + BX > d.N && d.n0 < d.N) d.flags |= 1;
+    const bool last_col = ((a.row_swap >> r) & 1) ? d.n0 + BX > gp.N : d.N == gp.N;   // the GEMM's last column tile
+    if ((gp.N & 7) != 0 && last_col && d.n0 < gp.N) d.flags |= 1;
     if ((a.row_swap >> r) & 1) d.flags |= kFlagSwap;
     a.tiles[k] = d;
   }

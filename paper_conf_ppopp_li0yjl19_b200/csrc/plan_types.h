@@ -49,15 +49,50 @@ constexpr int kF32MapsPerGemm = 2;
 struct alignas(16) TileDesc {
   int32_t gemm;
   int32_t m0;        // element row of the tile origin    (Y_Coord * BY)
-  int32_t n0;        // element column of the tile origin (X_Coord * BX)
+  int32_t n0;        // element column of the tile origin (balanced: see tile_cols below)
   int32_t kblocks;   // ceil(K / 64)
-  int32_t M, N;      // GEMM extents
+  int32_t M;         // GEMM rows
+  int32_t N;         // end column of the tile (the GEMM's N for its last column tile)
   int32_t ldc;       // elements
   uint16_t geo;      // (BY / 16) | (BX / 16) << 8
   uint16_t flags;    // bit 0: the tile's last C chunk ends inside a 16-byte granule (N % 8 != 0):
                      //        its columns [N & ~7, N) are stored directly, not by TMA
                      // bits 8-10: K=16 MMA steps of the last k-block (1..4), 0 = 4
 };
+// Balanced column split of a tensor-core GEMM (reading C-26): the ceil(N / BX) column
+// tiles of a GEMM share its ceil(N / G) column chunks (G = 64, or BX when narrower) as evenly as
+// whole chunks allow, instead of BX columns each plus a ragged last tile.  Tiles that share an A
+// row panel then stream it at the same speed, so its re-reads hit in L2 (a 256-column edge tile
+// of a 768-wide GEMM beside a 512-column one ran twice as fast and re-read A from DRAM).  The
+// plan (tile (y, x), Eq. 1 counts) is unchanged; chunk boundaries stay 64-column aligned, so no
+// TMA store box crosses into a neighbouring tile.  Returns [n0, end) of column tile x.
+#ifndef VB_BALANCED_N
+#define VB_BALANCED_N 1
+#endif
+__host__ __device__ inline void tile_cols(int x, int N, int BX, int &n0, int &end) {
+#if VB_BALANCED_N
+  const int G = BX < 64 ? BX : 64;
+  const int q = (N + G - 1) / G, nx = (N + BX - 1) / BX;
+  n0 = (int)((int64_t)x * q / nx) * G;
+  end = (int)((int64_t)(x + 1) * q / nx) * G;
+  if (end > N) end = N;
+#else
+  n0 = x * BX;
+  end = n0 + BX < N ? n0 + BX : N;
+#endif
+}
+// inverse of tile_cols: the column tile whose range starts at n0 (q >= nx, so n0 is strictly
+// increasing in x)
+__host__ __device__ inline int tile_col_index(int n0, int N, int BX) {
+#if VB_BALANCED_N
+  const int G = BX < 64 ? BX : 64;
+  const int q = (N + G - 1) / G, nx = (N + BX - 1) / BX;
+  return (int)(((int64_t)(n0 / G) * nx + q - 1) / q);
+#else
+  return n0 / BX;
+#endif
+}
+
 // Tensor maps per GEMM (128 bytes each): A, A row-tail, B, B K-tail, C (loads), C store.  The
 // tail maps have boxes that stop at the matrix edge, because out-of-bounds box rows are
 // zero-filled but still cost L2 request bandwidth.  The C store map is N & ~7 columns wide:
