@@ -56,6 +56,9 @@ constexpr int kPageBytes = 8192;
 #ifndef VB_KB_PREFETCH
 #define VB_KB_PREFETCH 0   // experiment: L2 prefetch of each A/B box this many k-blocks ahead
 #endif
+#ifndef VB_JIT_CLAIM
+#define VB_JIT_CLAIM 1   // pair kernel: claim each block just in time (reading C-27)
+#endif
 #ifndef VB_EPI_FFMA2
 #define VB_EPI_FFMA2 1   // epilogue alpha*acc + beta*C_old as paired fp32 FMUL2/FFMA2 (0: scalar)
 #endif
@@ -432,19 +435,28 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     // Software-pipelined by one block: while the tiles of block b are read and pushed, the
     // CSR range of the next block (claimed one ahead) is already in flight and the block after
     // it is being claimed, so each block costs one dependent global round trip, not three.
+    //
+    // The pair kernel (kJitClaim) instead claims each block just in time: after pushing a block
+    // it waits for the lookahead budget and only then claims the next one (reading C-27).  Its
+    // blocks hold long tiles (tens of microseconds); a block claimed two ahead starts up to two
+    // block durations after its claim, so the tiles of one GEMM -- claimed back to back by
+    // different pairs -- would start that far apart and re-read their shared A / B panels from
+    // DRAM.  The claim's two round trips (counter, block range) hide behind the kKbAhead k-blocks
+    // already pushed.
+    constexpr bool kJitClaim = PAIR && VB_JIT_CLAIM;
     int b = (int)blockIdx.x / (PAIR ? 2 : 1);
     int lim = (b < p.n_blocks && lane < 2) ? p.block_ptr[b + lane] : 0;
     int nb = 0;
-    if (lane == 0) nb = n_static + atomicAdd(p.counter, 1);
+    if (!kJitClaim && lane == 0) nb = n_static + atomicAdd(p.counter, 1);
     nb = __shfl_sync(0xffffffffu, nb, 0);
     for (;;) {
       if (b >= p.n_blocks) break;
       int nb2 = nb;
-      if (lane == 0) {
+      if (!kJitClaim && lane == 0) {
         VB_TWAIT(T_SCHED_BUDGET, while ((int)(pushed_kb - atomicAdd(&sh->prod_kb, 0u)) > kKbAhead) __nanosleep(128));
         if (nb < p.n_blocks) nb2 = n_static + atomicAdd(p.counter, 1);   // claim two ahead
       }
-      const int lim_next = (nb < p.n_blocks && lane < 2) ? p.block_ptr[nb + lane] : 0;
+      int lim_next = (!kJitClaim && nb < p.n_blocks && lane < 2) ? p.block_ptr[nb + lane] : 0;
       const int s0 = __shfl_sync(0xffffffffu, lim, 0), s1 = __shfl_sync(0xffffffffu, lim, 1);
       for (int base = s0; base < s1; base += 32) {
         const int n = min(32, s1 - base);
@@ -481,9 +493,20 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         pushed_kb += (uint32_t)kb;
         t += (uint32_t)n;
       }
-      b = nb;
-      lim = lim_next;
-      nb = __shfl_sync(0xffffffffu, nb2, 0);
+      if (kJitClaim) {
+        if (lane == 0) {
+          VB_TWAIT(T_SCHED_BUDGET, while ((int)(pushed_kb - atomicAdd(&sh->prod_kb, 0u)) > kKbAhead) __nanosleep(128));
+          nb = n_static + atomicAdd(p.counter, 1);
+        }
+        nb = __shfl_sync(0xffffffffu, nb, 0);
+        lim_next = (nb < p.n_blocks && lane < 2) ? p.block_ptr[nb + lane] : 0;
+        b = nb;
+        lim = lim_next;
+      } else {
+        b = nb;
+        lim = lim_next;
+        nb = __shfl_sync(0xffffffffu, nb2, 0);
+      }
     }
     if (lane == 0) {                                        // end marker
       const int e = (int)(t % kRing);

@@ -45,7 +45,8 @@ for b, m, n, k in [(4096, 128, 256, 1024), (16384, 256, 256, 256), (16384, 200, 
 # scripts/cublas_context.py)
 for b, m, n, k in [(64, 1024, 1024, 4096), (16, 2048, 2048, 4096), (256, 512, 512, 2048), (64, 1024, 1024, 1024),
                    (64, 1024, 1024, 256), (64, 1024, 1024, 512), (64, 1024, 1024, 2048), (256, 512, 512, 512),
-                   (256, 512, 512, 1024), (256, 512, 512, 4096), (400, 768, 768, 2048), (400, 1000, 1000, 2000)]:
+                   (256, 512, 512, 1024), (256, 512, 512, 4096), (400, 768, 768, 2048), (400, 1000, 1000, 2000),
+                   (400, 700, 1024, 2048), (400, 300, 1024, 2048), (400, 600, 700, 1500)]:
     cases[f"c{b}x{m}x{n}x{k}"] = (np.full(b, m), np.full(b, n), np.full(b, k))
 for k in (16, 32, 40, 48, 56, 64, 72, 100, 128, 200, 256):
     cases[f"K{k}"] = (np.full(32768, 128), np.full(32768, 256), np.full(32768, k))

@@ -7,7 +7,7 @@ out=${1:-gpurun_out/sanitizer}
 mkdir -p "$out"
 CS=/usr/local/cuda/bin/compute-sanitizer
 for tool in ${VB_SAN_TOOLS:-memcheck synccheck racecheck}; do
-  for c in c1 ragged_bf16 ragged_f32 pair conv graph; do
+  for c in ${VB_SAN_CASES:-c1 ragged_bf16 ragged_f32 pair w2 conv graph}; do
     timeout ${VB_SAN_TIMEOUT:-300} $CS --tool $tool --print-limit 20 --error-exitcode 9 --target-processes all \
       python tests/tools/sanitize_cases.py $c > "$out/${tool}_${c}.log" 2>&1
     echo "$tool $c rc=$? $(grep -h 'ERROR SUMMARY' "$out/${tool}_${c}.log" | tail -1) $(grep -h 'parity ok' "$out/${tool}_${c}.log")"

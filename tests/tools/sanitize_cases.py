@@ -5,7 +5,8 @@ proves the instrumented kernels still compute the right thing.
     compute-sanitizer --tool memcheck python tests/tools/sanitize_cases.py [case ...]
 
 cases: c1 (C1 fp32, 3 policies), ragged_bf16 / ragged_f32 (48 GEMMs, M, N, K in [1, 600]),
-pair (2-SM cta_group::2 tiles + 1-SM tiles, two GEMM launches), conv (GoogleNet 3a implicit
+pair (2-SM cta_group::2 tiles incl. W2 + 1-SM tiles, two GEMM launches), w2 (W2 / H2 pair tiles
+forced on ragged shapes: both MMA halves, N tails inside either half, K = 0), conv (GoogleNet 3a implicit
 GEMM, TMA im2col), graph (vb_exec_bound captured in a CUDA graph, 3 replays).
 """
 import os
@@ -65,6 +66,24 @@ def case_pair():
     K = np.array([1024, 700, 900, 1000, 600])
     plan = _run(M, N, K, "bf16", 0, thr=1)
     assert plan.info()["launches_per_exec"] == 3, plan.info()
+
+
+def case_w2():
+    from oracle import plan_ref as pr
+    N = np.array([512, 300, 260, 289, 511, 700, 1000, 257, 640, 768])
+    M = np.array([256, 300, 129, 512, 255, 384, 777, 256, 130, 17])
+    K = np.array([64, 100, 700, 0, 300, 150, 17, 640, 300, 1])
+    db = DeviceBatch(M, N, K, "bf16")
+    db.C.fill_(float("nan"))
+    db.fill(SEED)
+    rows = [15 if g % 3 else 10 for g in range(len(M))]
+    tiles = pr.enumerate_tiles(db.M, db.N, db.K, rows, pr.B200_TC)
+    plan = vb.plan_from_schedule(db.M, db.N, db.K, db.lda, db.ldb, db.ldc, rows, 256, list(range(len(tiles) + 1)),
+                                 [t.gemm for t in tiles], [t.y for t in tiles], [t.x for t in tiles], dtype="bf16",
+                                 device=0, table_id=3)
+    db.run(plan)
+    torch.cuda.synchronize()
+    check_batch(db, range(db.batch), SEED, "random")
 
 
 def case_conv():
