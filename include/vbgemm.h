@@ -66,7 +66,7 @@ typedef enum {
  *  VB_TABLE_B200_FFMA   Table 2 shapes without 128x128 (16x16 ... 128x64 / 64x128) with the
  *                       128-thread sub-tiles for the fp32 FFMA kernel, T = 128, B200 constants.
  *  VB_TABLE_B200_TC     tcgen05 table (bf16/fp16): 64x32, 128x32, 64x64, 128x64, 64x128,
- *                       128x128, 64x256, 128x256 C tiles and 2-SM pair tiles 256x{64,128,256},
+ *                       128x128, 64x256, 128x256 C tiles and 2-SM pair tiles 256x{64,128,256,512},
  *                       BK = 64, T = 256; availability tested against max(M, 128) x max(N, 256)
  *                       (reading C-1b).
  *  VB_TABLE_DEFAULT     B200_FFMA for VB_F32, B200_TC for VB_BF16 / VB_F16. */

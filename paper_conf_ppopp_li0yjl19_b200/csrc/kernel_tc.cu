@@ -4,12 +4,14 @@
 //
 // One CTA per SM (grid = min(Block_NUM, #SMs)), 16 warps:
 //   warp 0      scheduler: starts with block = CTA index, then claims blocks (work lists)
-//               with an atomic, software-pipelined one block ahead; loads their tile
+//               with an atomic, software-pipelined one block ahead (the pair kernel claims
+//               each block just in time, reading C-27); loads their tile
 //               descriptors (one 32-byte record per tile, lanes in parallel) into a 32-entry
 //               smem tile ring and prefetches the tiles' tensor maps; lookahead is bounded in
 //               k-blocks so the GPU works on a short window of GEMMs at a time (L2 reuse of A/B).
 //   warp 1      TMEM owner + MMA issuer: one thread issues tcgen05.mma (M = BY, N = BX,
-//               K = 16) into an accumulator ring of 512 TMEM columns (up to 8 tiles in flight).
+//               K = 16; a 256 x 512 W2 pair tile issues two N = 256 MMAs per K step) into an
+//               accumulator ring of 512 TMEM columns (up to 8 tiles in flight).
 //   warps 2-3   C_old producers: TMA-load C_old chunks (BY x 64) per epilogue quarter into a
 //               4-slot ring when beta != 0 (C is never read when beta == 0, reading C-16).
 //   warps 4-7   A/B producers: stream each tile's k-blocks (A: BY x 64, B: 64 x BX; for an
@@ -98,6 +100,14 @@ constexpr int kTmemCols = 512;
 constexpr int kAccUnit = 32;               // TMEM accumulator ring granularity (columns)
 constexpr int kAccUnits = kTmemCols / kAccUnit;
 constexpr int kAcc = 8;                    // accumulators in flight (ring entries)
+#ifndef VB_ACC_SPLIT
+#define VB_ACC_SPLIT 0   // experiment: accumulators of >= 8 units as two ring entries (halves)
+#endif
+// units of the first half of a split accumulator, 0 = not split (a half is whole 64-column
+// epilogue chunks, so the split point is a chunk boundary)
+__device__ __forceinline__ int split_units(int units) {
+  return (VB_ACC_SPLIT && units >= 8 && (units & 3) == 0) ? units / 2 : 0;
+}
 constexpr int kEpiWarps = 8;               // two per TMEM lane quarter, splitting each chunk's columns
 constexpr uint32_t kRingConsumers = kProducers + 1 + kCProducers + kEpiWarps;
 
@@ -443,7 +453,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
     // different pairs -- would start that far apart and re-read their shared A / B panels from
     // DRAM.  The claim's two round trips (counter, block range) hide behind the kKbAhead k-blocks
     // already pushed.
-    constexpr bool kJitClaim = PAIR && VB_JIT_CLAIM;
+    constexpr bool kJitClaim = (PAIR && VB_JIT_CLAIM) || VB_JIT_CLAIM == 2;
     int b = (int)blockIdx.x / (PAIR ? 2 : 1);
     int lim = (b < p.n_blocks && lane < 2) ? p.block_ptr[b + lane] : 0;
     int nb = 0;
@@ -702,16 +712,21 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         if (ti.d.gemm < 0) break;
         const int BY = geo_BY(ti.d.geo), BX = geo_BX(ti.d.geo);   // MMA shape (pair: M = 256)
         const TcGeom geo = tc_geom(PAIR ? BY / 2 : BY, PAIR ? min(BX, 256) / 2 : BX);   // this CTA's B half
-        const int e = (int)(t % kAcc);
-        ++t;
+        // VB_ACC_SPLIT: an accumulator of 8+ units is two ring entries (halves); the epilogue hands
+        // the first half back once drained, so a following tile that fits there starts early.
+        const int units = tile_acc_units(ti.d, PAIR, SWAP);
+        const int hu = split_units(units);
+        const int nent = hu ? 2 : 1;
+        const int e = (int)(t % kAcc), e1 = (int)((t + 1) % kAcc);
+        t += (uint32_t)nent;
 #ifdef VB_TRACE
         tr[T_TILES] += 1;
 #endif
         int take;
-        const int start = ring.place(tile_acc_units(ti.d, PAIR, SWAP), take);
+        const int start = ring.place(units, take);
         {
           VB_T0();
-          while (free_units < take || inflight == kAcc) {   // reclaim drained accumulators (FIFO)
+          while (free_units < take || inflight + nent > kAcc) {   // reclaim drained accumulators (FIFO)
             ptx::mbar_wait(&sh->tempty[oldest], ophase);
             free_units += acc_take[oldest];
             --inflight;
@@ -720,8 +735,13 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           VB_TADD(T_MMA_TEMPTY);
         }
         free_units -= take;
-        acc_take[e] = take;
-        ++inflight;
+        if (nent == 2) {   // entry e: the skipped ring end (if any) + the first half; e1: the rest
+          acc_take[e] = take - (units - hu);
+          acc_take[e1] = units - hu;
+        } else {
+          acc_take[e] = take;
+        }
+        inflight += nent;
         ptx::tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(start * kAccUnit);
         // swap-AB: A operand = the B panel (MN-major, M = BX = 128), B operand = the A rows
@@ -786,10 +806,13 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           advance(slot, sph, kSlots);
         }
         if (ptx::elect_lane0()) {
-          if (PAIR)
+          if (PAIR) {
             ptx::mma_commit_pair(&sh->tfull[e]);
-          else
+            if (nent == 2) ptx::mma_commit_pair(&sh->tfull[e1]);
+          } else {
             ptx::mma_commit(&sh->tfull[e]);         // accumulator ready for the epilogue
+            if (nent == 2) ptx::mma_commit(&sh->tfull[e1]);
+          }
           VB_STAMP(5);
         }
       }
@@ -878,11 +901,14 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
 #else
       const int n8 = ti.d.N & ~7;                       // the store map's width
 #endif
-      const int e = (int)(t % kAcc);
-      const uint32_t aph = (t / kAcc) & 1u;
-      ++t;
+      const int units = tile_acc_units(ti.d, PAIR, SWAP);
+      const int hu = split_units(units);                // the MMA warp's split, mirrored
+      const int nent = hu ? 2 : 1;
+      const int e = (int)(t % kAcc), e1 = (int)((t + 1) % kAcc);
+      const uint32_t aph = (t / kAcc) & 1u, aph1 = ((t + 1) / kAcc) & 1u;
+      t += (uint32_t)nent;
       int take;
-      const int acc_col = acc_ring.place(tile_acc_units(ti.d, PAIR, SWAP), take) * kAccUnit;
+      const int acc_col = acc_ring.place(units, take) * kAccUnit;
       // M = 128: tile row 32q + i lives in TMEM lane 32q + i.
       // M = 64 : tile row 16q + i lives in TMEM lane 32q + i, i < 16 (half sub-partitions).
       const int rows_w = BY / 4;
@@ -897,6 +923,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       tr[T_EPI_HEAD] += clock64() - _head_t0;
 #endif
       VB_TWAIT(T_EPI_TFULL, ptx::mbar_wait(&sh->tfull[e], aph));
+      if (nent == 2) ptx::mbar_wait(&sh->tfull[e1], aph1);   // committed with e
       if (lane == 0) VB_STAMP(6);
       ptx::tc_fence_after();
 #ifdef VB_TRACE
@@ -910,16 +937,17 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         else
           ptx::tmem_ld_32x32b_x16(ta, acc);
       };
-      auto release_acc = [&]() {                       // accumulator drained: hand it back early
+      auto release_entry = [&](int ent) {              // accumulator (part) drained: hand it back early
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) {
           if (!PAIR || leader)
-            ptx::mbar_arrive(&sh->tempty[e]);
+            ptx::mbar_arrive(&sh->tempty[ent]);
           else
-            ptx::mbar_arrive_remote(ptx::mapa(&sh->tempty[e], 0));
+            ptx::mbar_arrive_remote(ptx::mapa(&sh->tempty[ent], 0));
         }
       };
+      auto release_acc = [&]() { release_entry(e); };
       if (SWAP && (ti.d.flags & kFlagSwap)) {
         // swap-AB tile: TMEM lane 32q + i holds C column n0 + 32q + i, TMEM column j holds C row
         // m0 + j.  Warp 8+q takes rows [0, nr/2), warp 12+q rows [nr/2, nr), eight at a time;
@@ -1044,7 +1072,8 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           VB_TWAIT(T_EPI_TLOAD, tload(ch, a0));
           VB_TWAIT(T_EPI_TMEM, ptx::tmem_ld_wait());
         }
-        if (ch + 1 == nch) VB_TWAIT(T_EPI_REL, release_acc());
+        if (nent == 2 && (ch + 1) * geo.c_cols == hu * kAccUnit) release_entry(e);   // first half drained
+        if (ch + 1 == nch) VB_TWAIT(T_EPI_REL, release_entry(nent == 2 ? e1 : e));
         VB_TWAIT(T_EPI_PROC, process(ch, a0));
       }
 #ifdef VB_TRACE
