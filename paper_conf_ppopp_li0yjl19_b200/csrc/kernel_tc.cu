@@ -89,10 +89,26 @@ constexpr int kPageBytes = 8192;
 #define VB_NGRAN 16
 #endif
 constexpr int kNGran = VB_NGRAN;          // MMA N granularity per CTA for edge tiles (power of 2)
-constexpr int kPages = VB_PAGES;           // 144 KB of A/B staging (default)
+#ifndef VB_PAGES_PAIR
+#define VB_PAGES_PAIR VB_PAGES
+#endif
+#ifndef VB_CSLOTS_PAIR
+#define VB_CSLOTS_PAIR VB_CSLOTS
+#endif
+// Shared-memory split between the A/B page ring and the C slots, per kernel (experiment switches
+// VB_PAGES_PAIR / VB_CSLOTS_PAIR give the pair kernel its own split; by default both kernels use
+// 18 pages + 4 C slots).
+template <bool PAIR> struct Layout {
+  static constexpr int kPages = PAIR ? VB_PAGES_PAIR : VB_PAGES;
+  static constexpr int kCSlots = PAIR ? VB_CSLOTS_PAIR : VB_CSLOTS;
+  // a layout at the 227 KB opt-in limit has no alignment slack: the kernel then checks that
+  // dynamic shared memory starts 1024-byte aligned (SW128 atoms) and traps if not
+  static constexpr int kSlack = (kPages * 8192 + kCSlots * 16384 + 4096 > 232448 - 1024) ? 0 : 1024;
+};
 constexpr int kSlots = 16;                 // k-blocks in flight (bounded by pages anyway)
-constexpr int kCSlots = VB_CSLOTS;
-static_assert(kCSlots >= 2, "the epilogue defers each store's completion by one chunk: one C slot deadlocks");
+constexpr int kCSlotsMax = VB_CSLOTS > VB_CSLOTS_PAIR ? VB_CSLOTS : VB_CSLOTS_PAIR;
+static_assert(VB_CSLOTS >= 2 && VB_CSLOTS_PAIR >= 2,
+              "the epilogue defers each store's completion by one chunk: one C slot deadlocks");
 constexpr int kCSlotBytes = 128 * 128;     // BY rows x 128 B
 constexpr int kRing = 32;                  // tile-descriptor ring entries
 constexpr int kKbAhead = VB_KBAHEAD;       // scheduler lookahead budget in k-blocks (L2 locality)
@@ -148,7 +164,7 @@ __device__ __forceinline__ void vb_stamp(long long *buf, int i) {
 struct Shared {
   uint64_t full[kSlots], empty[kSlots];
   uint64_t tfull[kAcc], tempty[kAcc];
-  uint64_t cfull[kCSlots], cempty[kCSlots];
+  uint64_t cfull[kCSlotsMax], cempty[kCSlotsMax];
   uint64_t rfull[kRing], rempty[kRing];
   int32_t slot_page[kSlots];
   int32_t slot_pages[kProducers][kSlots];   // per producer replica: pages charged per k-block
@@ -158,8 +174,12 @@ struct Shared {
   TileInfo ring[kRing];
 };
 
-constexpr size_t kSmemBytes = 1024 /*align slack*/ + (size_t)kPages * kPageBytes + (size_t)kCSlots * kCSlotBytes +
-                              ((sizeof(Shared) + 127) / 128) * 128;
+template <bool PAIR>
+constexpr size_t smem_bytes() {
+  return (size_t)Layout<PAIR>::kSlack + (size_t)Layout<PAIR>::kPages * kPageBytes +
+         (size_t)Layout<PAIR>::kCSlots * kCSlotBytes + ((sizeof(Shared) + 127) / 128) * 128;
+}
+static_assert(smem_bytes<true>() <= 232448 && smem_bytes<false>() <= 232448, "over the 227 KB opt-in limit");
 
 // Opt-in cycle accounting (build with -DVB_TRACE): per-CTA cycles each role spends waiting
 // on each barrier, accumulated into TcArgs::trace[kTraceSlots] (unused in product builds).
@@ -352,7 +372,9 @@ __device__ __forceinline__ void epi_row(uint8_t *cb, int row, int c_swz, int u0,
 // owns the barriers both CTAs' TMA loads and epilogues report to.
 template <int AB_FMT, bool PAIR, bool SWAP = false>
 __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constant__ TcArgs p) {
+  constexpr int kPages = Layout<PAIR>::kPages, kCSlots = Layout<PAIR>::kCSlots;
   extern __shared__ uint8_t smem_raw[];
+  if (Layout<PAIR>::kSlack == 0 && (ptx::smem_u32(smem_raw) & 1023u) != 0u) __trap();
   // 1024-byte aligned (SW128 atoms); offsetting smem_raw itself keeps the shared address space
   // visible to the compiler, so C-slot and barrier accesses compile to LDS/STS, not generic LD/ST.
   uint8_t *smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
@@ -1159,15 +1181,15 @@ __global__ void vb_tc_prep(uint8_t *tmaps, const void *const *A, const void *con
 VB_COV_SETTER(tc_set_coverage)
 #endif
 
-size_t tc_smem_bytes() { return tck::kSmemBytes; }
+size_t tc_smem_bytes() { return tck::smem_bytes<false>(); }
 
 cudaError_t tc_configure() {
   cudaError_t e = cudaSuccess;
-  const int smem = (int)tck::kSmemBytes;
+  const int smem = (int)tck::smem_bytes<false>(), smem2 = (int)tck::smem_bytes<true>();
   if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(tck::vb_tc_kernel<0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(tck::vb_tc_kernel<1, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess)
@@ -1188,7 +1210,7 @@ cudaError_t launch_tc(const TcArgs &args, int grid, bool bf16, bool pair, bool s
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3(tck::kThreads);
-  cfg.dynamicSmemBytes = tck::kSmemBytes;
+  cfg.dynamicSmemBytes = pair ? tck::smem_bytes<true>() : tck::smem_bytes<false>();
   cfg.stream = stream;
   cudaLaunchAttribute attr[2];
   int na = 0;
