@@ -245,6 +245,15 @@ vb_status vb_plan_export(vb_plan_t plan, int32_t *block_ptr, int32_t *tile_gemm,
  * Errors: VB_ERR_INVALID_ARG (null plan, buffer too small), VB_ERR_CUDA. */
 vb_status vb_plan_debug_tmaps(vb_plan_t plan, void *out, int64_t bytes, int64_t *needed);
 
+/* vb_debug_tile_cols — diagnostic: the column range [*n0, *end) that column tile x of a
+ * tensor-core GEMM with N columns and strategy width BX covers in the kernels (DESIGN.md reading
+ * C-26: the GEMM's ceil(N / G) column chunks, G = min(64, BX), shared as evenly as whole chunks
+ * allow among its ceil(N / BX) column tiles), and *x_back = the tile index the plan export
+ * decodes from *n0.  Host only, no GPU needed.
+ * Errors: VB_ERR_INVALID_ARG (null outputs, N < 1, BX not a multiple of 16 in [16, 512],
+ * x outside [0, ceil(N / BX))). */
+vb_status vb_debug_tile_cols(int32_t x, int32_t N, int32_t BX, int32_t *n0, int32_t *end, int32_t *x_back);
+
 /* vb_debug_set_coverage — diagnostic, coverage-counter build only (libvbgemm_cov.so, compiled
  * with -DVB_COVERAGE; SURVEY.md §4 "each C element written exactly once"): from now on every
  * element a GEMM kernel's epilogue stores on `device` also adds 1 to the int32 counter at the

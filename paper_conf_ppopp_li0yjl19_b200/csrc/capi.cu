@@ -951,6 +951,19 @@ extern "C" vb_status vb_plan_info(vb_plan_t p, int64_t *n_tiles, int64_t *n_bloc
   return VB_OK;
 }
 
+extern "C" vb_status vb_debug_tile_cols(int32_t x, int32_t N, int32_t BX, int32_t *n0, int32_t *end,
+                                        int32_t *x_back) {
+  if (!n0 || !end || !x_back) return fail(VB_ERR_INVALID_ARG, "null output");
+  if (N < 1 || BX < 16 || BX > 512 || BX % 16) return fail(VB_ERR_INVALID_ARG, "bad N / BX");
+  if (x < 0 || x >= (N + BX - 1) / BX) return fail(VB_ERR_INVALID_ARG, "tile index out of range");
+  int a = 0, b = 0;
+  tile_cols(x, N, BX, a, b);
+  *n0 = a;
+  *end = b;
+  *x_back = tile_col_index(a, N, BX);
+  return VB_OK;
+}
+
 extern "C" vb_status vb_debug_set_coverage(int device, int32_t *counts, const void *c_base, int32_t elem_bytes) {
 #ifdef VB_COVERAGE
   DeviceGuard g(device);

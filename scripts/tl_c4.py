@@ -1,3 +1,7 @@
+"""Per-CTA exit spread of C4's two launches (pair launch: GEMMs with M >= 256; 1-SM launch: the
+rest), measurement tool; needs the -DVB_TIMELINE_ALL build:
+    python paper_conf_ppopp_li0yjl19_b200/build.py -DVB_TIMELINE_ALL --out=libvbgemm_ctatl.so
+    VB_LIB=paper_conf_ppopp_li0yjl19_b200/libvbgemm_ctatl.so python scripts/tl_c4.py"""
 import ctypes, os, sys
 sys.path.insert(0, os.getcwd())
 import numpy as np, torch, vbinputs

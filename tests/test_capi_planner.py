@@ -199,3 +199,31 @@ def test_conv_plan_validation_on_host():
     with pytest.raises(vb.VbError):
         nv.plan_conv([good], "f32", device=-1)
     assert nv.plan_conv([], "bf16", device=-1).info()["n_tiles"] == 0
+
+
+def test_balanced_column_split_c26():
+    """Reading C-26 through the product's own function (vb_debug_tile_cols): the column tiles of
+    a GEMM cover [0, N) exactly once, in order, every interior boundary 64-column aligned (no TMA
+    store box crosses into a neighbour), no tile wider than BX, widths within one chunk of each
+    other, and the export decodes each tile's index back from its origin."""
+    import ctypes
+    f = nv.lib.vb_debug_tile_cols
+    f.argtypes = [ctypes.c_int32] * 3 + [ctypes.POINTER(ctypes.c_int32)] * 3
+    a, b, xb = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    for BX in (32, 64, 128, 256, 512):
+        G = min(64, BX)
+        for N in list(range(1, 1100, 7)) + [BX, 2 * BX, 3 * BX - 1, 768, 700, 4096, 4097]:
+            nx = -(-N // BX)
+            prev, widths = 0, []
+            for x in range(nx):
+                assert f(x, N, BX, ctypes.byref(a), ctypes.byref(b), ctypes.byref(xb)) == vb.VB_OK
+                assert a.value == prev and b.value > a.value and b.value - a.value <= BX, (BX, N, x)
+                assert a.value % G == 0 and (b.value == N or b.value % G == 0), (BX, N, x)
+                assert xb.value == x
+                widths.append(b.value - a.value)
+                prev = b.value
+            assert prev == N
+            full = widths[:-1] if N % G else widths
+            assert not full or max(full) - min(full) <= G, (BX, N, widths)
+    assert f(1, 100, 128, ctypes.byref(a), ctypes.byref(b), ctypes.byref(xb)) == vb.VB_ERR_INVALID_ARG
+    assert f(0, 100, 100, ctypes.byref(a), ctypes.byref(b), ctypes.byref(xb)) == vb.VB_ERR_INVALID_ARG
