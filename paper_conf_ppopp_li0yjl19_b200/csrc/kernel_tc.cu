@@ -621,6 +621,13 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const int a_pages = (BY * kBK * 2 + kPageBytes - 1) / kPageBytes;   // swap-AB tiles: 16-64 rows, 1 page
         const int b_span = Nh1 ? kHalfBBytes + Nh1 * kBK * 2 : Nh0 * kBK * 2;   // B panel bytes of this CTA
         const int need = a_pages + (b_span + kPageBytes - 1) / kPageBytes;
+        // per-tile constants of the k-loop (the loop body is on the page-release -> TMA-issue
+        // latency chain): transaction bytes of the A rows and the B box count of both CTAs, and
+        // the first column of each MMA half's B boxes in this CTA
+        const uint32_t a_tx = (uint32_t)((a_box_rows_of(0) + (PAIR ? a_box_rows_of(1) : 0)) * kBK * 2);
+        const uint32_t b_box_tx = (uint32_t)((b_boxes_of(0) + (PAIR ? b_boxes_of(1) : 0)) * geo.b_swz);
+        const int bcol0 = ti.d.n0 + (int)rank * Nh0, bcol1 = ti.d.n0 + 256 + (int)rank * Nh1;
+        const int bstep = geo.b_swz / 2;
         for (int kb = 0; kb < ti.d.kblocks; ++kb, ++kbg) {
           int start = head, take = need;
           if (start + need > kPages) {          // never wrap a k-block around the ring end
@@ -652,15 +659,13 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           if (pid == 0) {
             sh->slot_page[slot] = start;
             if (leader) {                     // the leader's barrier counts both CTAs' bytes
-              uint32_t bytes = (uint32_t)(a_box_rows_of(0) * kBK * 2 + b_boxes_of(0) * b_rows * geo.b_swz);
-              if (PAIR) bytes += (uint32_t)(a_box_rows_of(1) * kBK * 2 + b_boxes_of(1) * b_rows * geo.b_swz);
-              ptx::mbar_arrive_expect_tx(&sh->full[slot], bytes);
+              ptx::mbar_arrive_expect_tx(&sh->full[slot], a_tx + b_box_tx * (uint32_t)b_rows);
               VB_STAMP(3);
             }
           }
           // box 0 = A, boxes 1..b_boxes = B; box i goes to producer (i + kbg) % kProducers
           if (ptx::elect_lane0())
-          for (int i = (int)((pid - kbg) % kProducers + kProducers) % kProducers; i <= b_boxes; i += kProducers) {
+          for (int i = (int)(((uint32_t)pid - kbg) % (uint32_t)kProducers); i <= b_boxes; i += kProducers) {
             if (i == 0 && a_box_rows == 0) continue;
             // B box i - 1: box j of half h (half 1 at kHalfBBytes, columns 256 on)
             const int h = i - 1 >= b_boxes0 ? 1 : 0, j = i - 1 - h * b_boxes0;
@@ -677,7 +682,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
               }
               continue;
             }
-            const int c0 = i == 0 ? kb * kBK : ti.d.n0 + h * 256 + (int)rank * (h ? Nh1 : Nh0) + j * (geo.b_swz / 2);
+            const int c0 = i == 0 ? kb * kBK : (h ? bcol1 : bcol0) + j * bstep;
             const int c1 = i == 0 ? row0 : kb * kBK;
             if (PAIR)
               ptx::tma_load_2d_pair(dst, map, &sh->full[slot], c0, c1);
