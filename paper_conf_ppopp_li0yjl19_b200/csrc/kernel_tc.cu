@@ -399,8 +399,10 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   // ordering (the TMEM reads are complete, nothing is published): the peer's epilogue warps
   // arrive on the leader's barrier with relaxed remote arrives.
   auto ring_release = [&](int e) { ptx::mbar_arrive(&sh->rempty[e]); };
+  // the leader's ring entries are written by its own scheduler (CTA scope); the peer's by the
+  // leader's scheduler through DSMEM (cluster scope)
   auto ring_wait = [&](int e, uint32_t ph) {
-    if (PAIR)
+    if (PAIR && !leader)
       ptx::mbar_wait_cluster(&sh->rfull[e], ph);
     else
       ptx::mbar_wait(&sh->rfull[e], ph);
