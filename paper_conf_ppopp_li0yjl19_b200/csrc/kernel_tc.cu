@@ -58,6 +58,9 @@ constexpr int kPageBytes = 8192;
 #ifndef VB_KB_PREFETCH
 #define VB_KB_PREFETCH 0   // experiment: L2 prefetch of each A/B box this many k-blocks ahead
 #endif
+#ifndef VB_PREFETCH_TAILS
+#define VB_PREFETCH_TAILS 1   // prefetch the tail maps a tile uses, and (pair) the peer SM's maps
+#endif
 #ifndef VB_JIT_CLAIM
 #define VB_JIT_CLAIM 1   // pair kernel: claim each block just in time (reading C-27)
 #endif
@@ -401,6 +404,23 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
   auto ring_release = [&](int e) { ptx::mbar_arrive(&sh->rempty[e]); };
   // the leader's ring entries are written by its own scheduler (CTA scope); the peer's by the
   // leader's scheduler through DSMEM (cluster scope)
+  // warm this SM's TMA descriptor cache for a tile's maps well before its producers use them
+  // (the row-tail and K-tail maps too, when the tile uses them: a tile's first k-block or its
+  // last one would otherwise wait for a descriptor fetch)
+  auto prefetch_tile_maps = [&](const TileDesc &d) {
+    const uint8_t *maps = reinterpret_cast<const uint8_t *>(p.tmaps) + (size_t)d.gemm * (kMapsPerGemm * 128);
+    if (d.kblocks > 0) {
+      ptx::prefetch_tmap(maps + MAP_A * 128);
+      ptx::prefetch_tmap(maps + MAP_B * 128);
+#if VB_PREFETCH_TAILS
+      const int BYc = geo_BY(d.geo) / (PAIR ? 2 : 1);
+      if (d.M % BYc != 0 && d.m0 + geo_BY(d.geo) > d.M) ptx::prefetch_tmap(maps + MAP_A_TAIL * 128);
+      if (!(d.flags & kFlagConv) && ((d.flags >> 8) & 7) != 0) ptx::prefetch_tmap(maps + MAP_B_TAIL * 128);
+#endif
+    }
+    ptx::prefetch_tmap(maps + MAP_C * 128);
+    if (d.N >= 8) ptx::prefetch_tmap(maps + MAP_C_ST * 128);
+  };
   auto ring_wait = [&](int e, uint32_t ph) {
     if (PAIR && !leader)
       ptx::mbar_wait_cluster(&sh->rfull[e], ph);
@@ -503,13 +523,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
           const TileDesc d = p.tiles[base + lane];
           kb = max(d.kblocks, 1);
           // warm the TMA descriptor cache for the tile's maps well before the producers use them
-          const uint8_t *maps = tmaps + (size_t)d.gemm * (kMapsPerGemm * 128);
-          if (d.kblocks > 0) {
-            ptx::prefetch_tmap(maps + MAP_A * 128);
-            ptx::prefetch_tmap(maps + MAP_B * 128);
-          }
-          ptx::prefetch_tmap(maps + MAP_C * 128);
-          if (d.N >= 8) ptx::prefetch_tmap(maps + MAP_C_ST * 128);
+          prefetch_tile_maps(d);
           const uint32_t tt = t + lane;
           const int e = (int)(tt % kRing);
           VB_TWAIT(T_SCHED_REMPTY, ptx::mbar_wait(&sh->rempty[e], ((tt / kRing) & 1u) ^ 1u));
@@ -566,6 +580,9 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         const uint32_t ph = (t / kRing) & 1u;
         ring_wait(e, ph);
         const bool end = sh->ring[e].d.gemm < 0;
+#if VB_PREFETCH_TAILS
+        if (!end) prefetch_tile_maps(sh->ring[e].d);   // the peer SM's own descriptor cache
+#endif
         ptx::mbar_wait(&sh->rempty[e], ph);
         ptx::mbar_arrive_remote(ptx::mapa(&sh->rempty[e], 0));
         if (end) break;
