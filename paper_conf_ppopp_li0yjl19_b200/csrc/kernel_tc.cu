@@ -120,12 +120,17 @@ constexpr int kAccUnit = 32;               // TMEM accumulator ring granularity 
 constexpr int kAccUnits = kTmemCols / kAccUnit;
 constexpr int kAcc = 8;                    // accumulators in flight (ring entries)
 #ifndef VB_ACC_SPLIT
-#define VB_ACC_SPLIT 0   // experiment: accumulators of >= 8 units as two ring entries (halves)
+#define VB_ACC_SPLIT 1   // 1: in the 1-SM kernel, 2: in both kernels, 0: off
 #endif
-// units of the first half of a split accumulator, 0 = not split (a half is whole 64-column
-// epilogue chunks, so the split point is a chunk boundary)
+// Accumulators of 8+ units as two ring entries (halves): the epilogue hands the first half back
+// as soon as it is drained, so a following tile that fits there starts its MMAs early.  Measured
+// (paired rounds): C5 0.99 (1-SM kernel, short-K tiles with 128-column neighbours), C4 1.015 when
+// also used by the pair kernel (its W2 neighbours rarely fit in a half) -- so 1-SM only.
+// Returns the units of the first half, 0 = not split (a half is whole 64-column epilogue chunks).
+template <bool PAIR>
 __device__ __forceinline__ int split_units(int units) {
-  return (VB_ACC_SPLIT && units >= 8 && (units & 3) == 0) ? units / 2 : 0;
+  const bool on = PAIR ? VB_ACC_SPLIT == 2 : VB_ACC_SPLIT != 0;
+  return (on && units >= 8 && (units & 3) == 0) ? units / 2 : 0;
 }
 constexpr int kEpiWarps = 8;               // two per TMEM lane quarter, splitting each chunk's columns
 constexpr uint32_t kRingConsumers = kProducers + 1 + kCProducers + kEpiWarps;
@@ -778,7 +783,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
         // VB_ACC_SPLIT: an accumulator of 8+ units is two ring entries (halves); the epilogue hands
         // the first half back once drained, so a following tile that fits there starts early.
         const int units = tile_acc_units(ti.d, PAIR, SWAP);
-        const int hu = split_units(units);
+        const int hu = split_units<PAIR>(units);
         const int nent = hu ? 2 : 1;
         const int e = (int)(t % kAcc), e1 = (int)((t + 1) % kAcc);
         t += (uint32_t)nent;
@@ -965,7 +970,7 @@ __global__ void __launch_bounds__(kThreads, 1) vb_tc_kernel(const __grid_constan
       const int n8 = ti.d.N & ~7;                       // the store map's width
 #endif
       const int units = tile_acc_units(ti.d, PAIR, SWAP);
-      const int hu = split_units(units);                // the MMA warp's split, mirrored
+      const int hu = split_units<PAIR>(units);                // the MMA warp's split, mirrored
       const int nent = hu ? 2 : 1;
       const int e = (int)(t % kAcc), e1 = (int)((t + 1) % kAcc);
       const uint32_t aph = (t / kAcc) & 1u, aph1 = ((t + 1) / kAcc) & 1u;
