@@ -309,6 +309,38 @@ def test_w2_tiles_forced(dtype):
     _padding_untouched(db)
 
 
+def test_pair_kernel_repeated_and_graph_replays():
+    """The pair kernel's cross-CTA protocol (mirrored tile ring, the peer's release forwarder,
+    relaxed accumulator releases, just-in-time claims) over repeated launches of one bound plan
+    and CUDA-graph replays: W2 + H2 + 1-SM tiles, beta != 0, every result checked."""
+    M = np.array([512, 300, 777, 1024, 100, 256, 640]); N = np.array([512, 260, 640, 1000, 96, 512, 700])
+    K = np.array([2048, 1500, 1900, 4096, 3000, 2000, 33])
+    db = DeviceBatch(M, N, K, "bf16")
+    db.fill(SEED)
+    c0 = db.C.clone()
+    plan = db.plan(tlp_threshold=1)
+    assert plan.info()["launches_per_exec"] == 3
+    db.bind(plan)
+    for _ in range(3):
+        db.C.copy_(c0)
+        db.run_bound(plan)
+        torch.cuda.synchronize()
+        check_batch(db, range(len(M)), SEED, "random")
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(s):
+        db.run_bound(plan, s)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=s):
+            db.run_bound(plan, s)
+    for _ in range(3):
+        db.C.copy_(c0)
+        torch.cuda.synchronize()
+        g.replay()
+        torch.cuda.synchronize()
+        check_batch(db, range(len(M)), SEED, "random")
+
+
 # ------------------------------------------------------------------ policy selection (P272-274)
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])
 def test_auto_policy_parity(dtype):
